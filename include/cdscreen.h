@@ -1,0 +1,168 @@
+/*
+ * cdscreen.h -- C ABI of the B200-native conjunction-screening library (libcdscreen.so).
+ *
+ * Implements the data-parallel screening path of Hellwig, Czappa, Michel, Bertrand, Wolf,
+ * "Satellite Collision Detection using Spatial Data Structures", IPDPS 2023:
+ * per sampling step, propagate every object, hash its position into a
+ * uniform grid of cell size g_c = d + 7.8 dt (Eq. 1) held in a non-blocking atomic
+ * hash map (Eq. 2), scan each occupied cell and its 26 neighbours (P:62, P:95,
+ * P:162), and refine every candidate's time and distance of closest approach with Brent's
+ * method.  The hybrid variant reuses the grid as a coarse
+ * pre-filter ahead of the apogee/perigee, orbit-path and time filters.
+ *
+ * Conventions for every call:
+ *   Units      km, s, rad.  All floating point is IEEE fp64.
+ *   Elements   osculating Kepler elements at epoch t = 0 (a, e, i, Omega, omega, true
+ *              anomaly), structure of arrays, n entries each, caller-owned, read-only, never
+ *              retained after the call returns.  Host pointers unless
+ *              cd_options.inputs_on_device != 0 (then device pointers on cd_options.device).
+ *   Steps      t_k = t0 + k dt (computed as fma(k, dt, t0)), k = 0 .. K-1,
+ *              K = floor((t1 - t0)/dt) + 1 (P:242-246 o = t/s_ps; both ends included).
+ *   Candidates (i, j, k), i < j, with |r_i(t_k) - r_j(t_k)| < g_c (strict).
+ *   Conjunctions  local minima of D(t) = |r_i(t) - r_j(t)| with D < d (strict) and TCA in
+ *              [t0, t1].  Each minimum is reported once, by its owner step
+ *              k = floor((TCA - t0)/dt + 1/2) (the step whose half-open cell
+ *              [t_k - dt/2, t_k + dt/2) contains it), and only if (i, j, k) is a candidate.
+ *   Output     sorted by (i, j, step), i < j; identical for any thread schedule and
+ *              independent of grid_origin and n_ranks (the union over ranks is the same set).
+ *   Ownership  outputs are library-owned until released with the matching *_free call.
+ *   Errors     every call returns cd_status; nothing throws across the ABI.  On error the output
+ *              is {NULL, 0} and cd_last_error() (thread-local) explains.  CUDA errors map to
+ *              CD_ECUDA with the driver's message.
+ *   Threads    calls may be made from several host threads; each call uses its own stream and
+ *              scratch memory.
+ */
+#ifndef CDSCREEN_H
+#define CDSCREEN_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CD_ABI_VERSION 1
+
+typedef enum {
+    CD_OK = 0,
+    CD_EINVAL = 1,    /* invalid argument (see validation rules below)                        */
+    CD_ENOMEM = 2,    /* device or host allocation failed even after capacity retries         */
+    CD_ECUDA = 3,     /* a CUDA runtime/driver error; cd_last_error() has the message          */
+    CD_ENCCL = 4,     /* reserved: collective failure (the merge runs in the Python layer)     */
+    CD_ERANGE = 5,    /* a position fell outside the key range +-(2^20 - 2) cells of g_c       */
+    CD_EINTERNAL = 6, /* internal invariant violated                                           */
+    CD_ENODEV = 7     /* no CUDA device / the library was not built for this device            */
+} cd_status;
+
+typedef enum {
+    CD_GRID = 0,   /* grid-based variant                               */
+    CD_HYBRID = 1  /* hybrid: coarse grid + orbital filter chain             */
+} cd_mode;
+
+/* Kepler elements, structure of arrays.  a > 0 [km], 0 <= e < 1, angles finite [rad]. */
+typedef struct {
+    const double* a;
+    const double* e;
+    const double* inc;
+    const double* raan;
+    const double* argp;
+    const double* nu0; /* true anomaly at epoch t = 0 */
+} cd_elements;
+
+/* conjunction flags */
+#define CD_FLAG_DEGENERATE 2u /* |v_i - v_j| < 1e-9 km/s at t_k: D stationary; tca = t_k, pca = D(t_k) */
+#define CD_FLAG_COPLANAR 4u   /* hybrid: pair took the coplanar (grid-refinement) path        */
+
+typedef struct {
+    uint32_t i, j;   /* object indices into the element arrays, i < j            */
+    uint32_t step;   /* owner step k                                              */
+    uint32_t flags;  /* CD_FLAG_*                                                 */
+    double tca;      /* time of closest approach [s from epoch]                   */
+    double pca;      /* distance at closest approach [km]                        */
+} cd_conjunction;    /* 32 B */
+
+typedef struct {
+    uint32_t i, j, step;
+} cd_candidate;      /* 12 B: the level-1 set (parity hook) */
+
+typedef struct {
+    cd_conjunction* data; /* host memory, or device memory if cd_options.outputs_on_device */
+    size_t count;
+    void* _owner;         /* library bookkeeping; do not touch */
+} cd_conjunctions;
+
+/* Per-call statistics (all optional outputs). */
+typedef struct {
+    uint64_t steps;            /* sampling steps screened by this call (this rank's slice)    */
+    uint64_t object_steps;     /* n * steps                                                    */
+    uint64_t candidates;       /* |K| for this slice (hybrid: coarse candidates)              */
+    uint64_t refined;          /* candidates that survived the conservative linear pre-filter
+                                  (hybrid: non-coplanar time-window work items + coplanar)    */
+    uint64_t conjunctions;     /* reported rows                                               */
+    uint64_t hybrid_ap_rejected, hybrid_coplanar, hybrid_path_rejected, hybrid_time_rejected;
+    uint64_t kernel_launches;  /* CUDA kernels launched by this call                          */
+    uint64_t retries;          /* capacity-overflow retries                                   */
+    double ms_total;           /* device time of the call (CUDA events on the call's stream)  */
+    double ms_propagate_insert, ms_scan, ms_refine, ms_finalize; /* per-phase device time (only
+                                  when cd_options.profile_phases != 0; adds syncs)            */
+} cd_stats;
+
+typedef struct {
+    double v_margin;          /* Eq. 1 speed [km/s]; default 7.8; 0 => cell = d               */
+    double grid_origin[3];    /* grid origin o [km]; default 0; results must not depend on it */
+    int device;               /* CUDA device ordinal; -1 = current                            */
+    void* stream;             /* cudaStream_t to run on; NULL = the library's own stream      */
+    int rank, n_ranks;        /* time slicing: this call screens steps
+                                 [floor(rank K / n_ranks), floor((rank+1) K / n_ranks));
+                                 default 0, 1                                                 */
+    int inputs_on_device;     /* element pointers are device pointers                         */
+    int outputs_on_device;    /* cd_conjunctions.data stays in device memory                  */
+    int kepler_points;        /* 0 = choose the Contour point count per object from e         */
+    double cell_factor;       /* grid cell edge = cell_factor * g_c (>= 1); default 1 (paper)  */
+    size_t batch_object_steps;/* object-steps per in-flight step batch; 0 = auto              */
+    size_t round_steps;       /* steps per refinement round; 0 = auto                         */
+    int profile_phases;       /* fill cd_stats per-phase times (serialises phases)            */
+    cd_stats* stats;          /* optional output                                              */
+} cd_options;
+
+/* Fill *opt with the defaults above. */
+void cd_options_init(cd_options* opt);
+
+/* Screen n objects over [t0, t1] at sampling step dt with threshold d.
+ * mode = CD_GRID:   g_c = d + v_margin*dt, candidates refined by Brent's method on
+ *                   [t_k - t_w, t_k + t_w], t_w = 2 g_c / min(|v_i|, |v_j|).
+ * mode = CD_HYBRID: same grid at the (coarse) dt given; candidates pass the apogee/perigee,
+ *                   coplanarity, orbit-path and time filters; survivors are refined inside
+ *                   their time windows.
+ * Validation (CD_EINVAL): elements non-NULL, 2 <= n < 2^32 - 1 (n = 0 or 1 returns an empty
+ * result), a > 0, 0 <= e < 1, finite angles, dt > 0, t1 >= t0, d > 0, K < 2^32,
+ * cell_factor >= 1, 0 <= rank < n_ranks.  out must be non-NULL. */
+cd_status cd_screen(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,
+                    cd_mode mode, cd_conjunctions* out);
+cd_status cd_screen_ex(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,
+                       cd_mode mode, const cd_options* opt /* nullable */, cd_conjunctions* out);
+
+/* The level-1 candidate set K for [t0, t1] at step dt with g_c = d + v_margin*dt
+ * (mode is accepted for symmetry; the set does not depend on it).  *out is a library-owned
+ * host array of *count entries sorted by (i, j, step); release with cd_candidates_free. */
+cd_status cd_candidates(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,
+                        cd_mode mode, const cd_options* opt, cd_candidate** out, size_t* count);
+
+/* Positions (and optionally velocities) of all n objects at nt times.  xyz (and vxyz, nullable)
+ * are caller-owned host buffers of nt*n*3 doubles, layout [time][object][x,y,z]. */
+cd_status cd_propagate(const cd_elements* el, size_t n, const double* t, size_t nt, double* xyz,
+                       double* vxyz, const cd_options* opt /* nullable */);
+
+void cd_conjunctions_free(cd_conjunctions* c);
+void cd_candidates_free(cd_candidate* c);
+const char* cd_status_str(cd_status s);
+const char* cd_last_error(void);
+int cd_abi_version(void);
+/* Total CUDA kernels launched by this process through the library (diagnostic). */
+uint64_t cd_kernel_launches(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CDSCREEN_H */

@@ -79,6 +79,9 @@ def lib():
         L.orc_pair_distance.restype = None
         L.orc_pair_distance.argtypes = [P(_Elements), C.c_int64, C.c_int64, P(C.c_double),
                                         C.c_int64, P(C.c_double), P(C.c_double)]
+        L.orc_candidate_flags.restype = None
+        L.orc_candidate_flags.argtypes = [P(_Elements), C.c_int64, C.c_double, C.c_double,
+                                          C.c_double, C.c_void_p, C.c_int64, C.c_void_p]
         L.orc_free.restype = None
         L.orc_free.argtypes = [C.c_void_p]
         if hasattr(L, "orc_hybrid"):
@@ -181,6 +184,16 @@ def conjunctions(pop, t0, t1, dt, d, gc, cands):
     c = lib().orc_conjunctions(P.ref, P.n, t0, t1, dt, d, gc, cands.ctypes.data_as(C.c_void_p),
                                cands.shape[0], C.byref(out))
     return _take(out, c, CONJ_DTYPE)
+
+
+def candidate_flags(pop, t0, dt, gc, cands):
+    """MULTI / DEGENERATE flags of arbitrary candidates (parity exclusions)."""
+    P = _Pop(pop)
+    cands = np.ascontiguousarray(cands, dtype=CAND_DTYPE)
+    f = np.zeros(cands.shape[0], dtype=np.uint32)
+    lib().orc_candidate_flags(P.ref, P.n, t0, dt, gc, cands.ctypes.data_as(C.c_void_p),
+                              cands.shape[0], f.ctypes.data_as(C.c_void_p))
+    return f
 
 
 def pair_distance(pop, i, j, times):

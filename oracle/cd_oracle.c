@@ -524,3 +524,36 @@ void orc_pair_distance(const orc_elements* el, int64_t i, int64_t j, const doubl
 }
 
 void orc_free(void* p) { free(p); }
+
+/* Flags of arbitrary candidates (test helper for parity exclusions): ORC_MULTI when g changes
+ * sign more than once on [t_k - t_w, t_k + t_w], ORC_DEGENERATE when |v_i - v_j| < 1e-9 km/s
+ * at t_k -- the same predicates orc_refine_one applies. */
+void orc_candidate_flags(const orc_elements* el, int64_t n, double t0, double dt, double gc,
+                         const orc_candidate* cand, int64_t ncand, uint32_t* flags)
+{
+    orc_orbit* o = orc_make_orbits(el, n);
+#pragma omp parallel for schedule(dynamic, 16)
+    for (int64_t q = 0; q < ncand; ++q) {
+        const orc_orbit* A = &o[cand[q].i];
+        const orc_orbit* B = &o[cand[q].j];
+        double tk = orc_step_time((int64_t)cand[q].step, t0, dt);
+        double ra[3], va[3], rb[3], vb[3];
+        orc_state(A, tk, ra, va);
+        orc_state(B, tk, rb, vb);
+        double dv2 = 0.0, sa = 0.0, sb = 0.0;
+        for (int c = 0; c < 3; ++c) {
+            dv2 += (va[c] - vb[c]) * (va[c] - vb[c]);
+            sa += va[c] * va[c];
+            sb += vb[c] * vb[c];
+        }
+        uint32_t f = 0;
+        if (sqrt(dv2) < 1e-9) {
+            f |= ORC_DEGENERATE;
+        } else {
+            double tw = 2.0 * gc / sqrt(fmin(sa, sb));
+            if (count_sign_changes(A, B, tk - tw, tk + tw, 64) > 1) f |= ORC_MULTI;
+        }
+        flags[q] = f;
+    }
+    free(o);
+}

@@ -1,0 +1,291 @@
+"""B200-native conjunction screening (Hellwig et al., IPDPS 2023) -- Python binding.
+
+Thin ctypes binding of ``libcdscreen.so`` (C ABI declared in ``include/cdscreen.h``).  This
+module only marshals arguments: every step of the screening path runs in the library's CUDA
+kernels.  There is no CPU fallback: if the extension is missing or no B200 is present, calls
+raise.
+
+The same names as the C ABI are exported (``cd_screen``, ``cd_screen_ex``, ``cd_candidates``,
+``cd_propagate``, ...) plus numpy-friendly wrappers ``screen``, ``candidates``, ``propagate``.
+"""
+from __future__ import annotations
+
+import ctypes as C
+from pathlib import Path
+
+import numpy as np
+
+PKG = Path(__file__).resolve().parent
+LIB_PATH = PKG / "libcdscreen.so"
+
+CD_OK, CD_EINVAL, CD_ENOMEM, CD_ECUDA, CD_ENCCL, CD_ERANGE, CD_EINTERNAL, CD_ENODEV = range(8)
+CD_GRID, CD_HYBRID = 0, 1
+CD_FLAG_DEGENERATE = 2
+CD_FLAG_COPLANAR = 4
+FIELDS = ("a", "e", "inc", "raan", "argp", "nu0")
+
+CONJ_DTYPE = np.dtype([("i", "<u4"), ("j", "<u4"), ("step", "<u4"), ("flags", "<u4"),
+                       ("tca", "<f8"), ("pca", "<f8")])
+CAND_DTYPE = np.dtype([("i", "<u4"), ("j", "<u4"), ("step", "<u4")])
+
+# C ABI symbols declared in include/cdscreen.h
+ABI_SYMBOLS = ("cd_options_init", "cd_screen", "cd_screen_ex", "cd_candidates", "cd_propagate",
+               "cd_conjunctions_free", "cd_candidates_free", "cd_status_str", "cd_last_error",
+               "cd_abi_version", "cd_kernel_launches")
+
+
+class CdError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{status_str(status)}: {msg}")
+        self.status = status
+
+
+class cd_elements(C.Structure):
+    _fields_ = [(k, C.c_void_p) for k in FIELDS]
+
+
+class cd_conjunction(C.Structure):
+    _fields_ = [("i", C.c_uint32), ("j", C.c_uint32), ("step", C.c_uint32), ("flags", C.c_uint32),
+                ("tca", C.c_double), ("pca", C.c_double)]
+
+
+class cd_candidate(C.Structure):
+    _fields_ = [("i", C.c_uint32), ("j", C.c_uint32), ("step", C.c_uint32)]
+
+
+class cd_conjunctions(C.Structure):
+    _fields_ = [("data", C.c_void_p), ("count", C.c_size_t), ("_owner", C.c_void_p)]
+
+
+class cd_stats(C.Structure):
+    _fields_ = [("steps", C.c_uint64), ("object_steps", C.c_uint64), ("candidates", C.c_uint64),
+                ("refined", C.c_uint64), ("conjunctions", C.c_uint64),
+                ("hybrid_ap_rejected", C.c_uint64), ("hybrid_coplanar", C.c_uint64),
+                ("hybrid_path_rejected", C.c_uint64), ("hybrid_time_rejected", C.c_uint64),
+                ("kernel_launches", C.c_uint64), ("retries", C.c_uint64),
+                ("ms_total", C.c_double), ("ms_propagate_insert", C.c_double),
+                ("ms_scan", C.c_double), ("ms_refine", C.c_double), ("ms_finalize", C.c_double)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class cd_options(C.Structure):
+    _fields_ = [("v_margin", C.c_double), ("grid_origin", C.c_double * 3), ("device", C.c_int),
+                ("stream", C.c_void_p), ("rank", C.c_int), ("n_ranks", C.c_int),
+                ("inputs_on_device", C.c_int), ("outputs_on_device", C.c_int),
+                ("kepler_points", C.c_int), ("cell_factor", C.c_double),
+                ("batch_object_steps", C.c_size_t), ("round_steps", C.c_size_t),
+                ("profile_phases", C.c_int), ("stats", C.POINTER(cd_stats))]
+
+
+_lib = None
+
+
+def lib():
+    """Load libcdscreen.so (built in-tree by __graft_entry__.build()).  Fails loudly."""
+    global _lib
+    if _lib is None:
+        if not LIB_PATH.exists():
+            raise ImportError(f"{LIB_PATH} is missing: run `python -c 'import __graft_entry__ as g; "
+                              f"g.build()'` (nvcc, sm_100a) -- there is no CPU fallback")
+        L = C.CDLL(str(LIB_PATH))
+        P = C.POINTER
+        L.cd_options_init.restype = None
+        L.cd_options_init.argtypes = [P(cd_options)]
+        L.cd_screen.restype = C.c_int
+        L.cd_screen.argtypes = [P(cd_elements), C.c_size_t, C.c_double, C.c_double, C.c_double,
+                                C.c_double, C.c_int, P(cd_conjunctions)]
+        L.cd_screen_ex.restype = C.c_int
+        L.cd_screen_ex.argtypes = [P(cd_elements), C.c_size_t, C.c_double, C.c_double, C.c_double,
+                                   C.c_double, C.c_int, P(cd_options), P(cd_conjunctions)]
+        L.cd_candidates.restype = C.c_int
+        L.cd_candidates.argtypes = [P(cd_elements), C.c_size_t, C.c_double, C.c_double, C.c_double,
+                                    C.c_double, C.c_int, P(cd_options), P(C.c_void_p),
+                                    P(C.c_size_t)]
+        L.cd_propagate.restype = C.c_int
+        L.cd_propagate.argtypes = [P(cd_elements), C.c_size_t, C.c_void_p, C.c_size_t, C.c_void_p,
+                                   C.c_void_p, P(cd_options)]
+        L.cd_conjunctions_free.restype = None
+        L.cd_conjunctions_free.argtypes = [P(cd_conjunctions)]
+        L.cd_candidates_free.restype = None
+        L.cd_candidates_free.argtypes = [C.c_void_p]
+        L.cd_status_str.restype = C.c_char_p
+        L.cd_status_str.argtypes = [C.c_int]
+        L.cd_last_error.restype = C.c_char_p
+        L.cd_abi_version.restype = C.c_int
+        L.cd_kernel_launches.restype = C.c_uint64
+        _lib = L
+    return _lib
+
+
+def status_str(s: int) -> str:
+    return lib().cd_status_str(s).decode()
+
+
+def last_error() -> str:
+    return lib().cd_last_error().decode()
+
+
+def _check(s):
+    if s != CD_OK:
+        raise CdError(s, last_error())
+
+
+# raw C-ABI names -------------------------------------------------------------------------
+def cd_options_init(opt):
+    lib().cd_options_init(C.byref(opt))
+
+
+def cd_screen(el, n, t0, t1, dt, d, mode, out):
+    return lib().cd_screen(C.byref(el), n, t0, t1, dt, d, mode, C.byref(out))
+
+
+def cd_screen_ex(el, n, t0, t1, dt, d, mode, opt, out):
+    return lib().cd_screen_ex(C.byref(el), n, t0, t1, dt, d, mode,
+                              C.byref(opt) if opt is not None else None, C.byref(out))
+
+
+def cd_candidates(el, n, t0, t1, dt, d, mode, opt, out, count):
+    return lib().cd_candidates(C.byref(el), n, t0, t1, dt, d, mode,
+                               C.byref(opt) if opt is not None else None, C.byref(out),
+                               C.byref(count))
+
+
+def cd_propagate(el, n, t, nt, xyz, vxyz, opt):
+    return lib().cd_propagate(C.byref(el), n, t, nt, xyz, vxyz,
+                              C.byref(opt) if opt is not None else None)
+
+
+def cd_conjunctions_free(c):
+    lib().cd_conjunctions_free(C.byref(c))
+
+
+def cd_candidates_free(p):
+    lib().cd_candidates_free(p)
+
+
+def cd_abi_version() -> int:
+    return lib().cd_abi_version()
+
+
+def cd_kernel_launches() -> int:
+    return int(lib().cd_kernel_launches())
+
+
+# numpy / torch wrappers --------------------------------------------------------------------
+class _Elements:
+    """Holds the arrays alive while the C call runs.  numpy -> host pointers; torch CUDA
+    tensors -> device pointers (inputs_on_device)."""
+
+    def __init__(self, pop):
+        first = pop["a"]
+        self.on_device = hasattr(first, "is_cuda") and bool(first.is_cuda)
+        if self.on_device:
+            self.keep = [pop[k].contiguous() for k in FIELDS]
+            ptrs = [t.data_ptr() for t in self.keep]
+            self.n = int(self.keep[0].numel())
+        else:
+            self.keep = [np.ascontiguousarray(np.asarray(pop[k], dtype=np.float64)) for k in FIELDS]
+            ptrs = [a.ctypes.data for a in self.keep]
+            self.n = int(self.keep[0].shape[0])
+        self.s = cd_elements(*ptrs)
+
+
+def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None, stream=None,
+                 cell_factor=None, batch_object_steps=None, round_steps=None,
+                 outputs_on_device=False, inputs_on_device=False):
+    o = cd_options()
+    cd_options_init(o)
+    o.rank, o.n_ranks = rank, n_ranks
+    if v_margin is not None:
+        o.v_margin = v_margin
+    if grid_origin is not None:
+        for c in range(3):
+            o.grid_origin[c] = float(grid_origin[c])
+    if device is not None:
+        o.device = int(device)
+    if stream is not None:
+        o.stream = stream
+    if cell_factor is not None:
+        o.cell_factor = float(cell_factor)
+    if batch_object_steps is not None:
+        o.batch_object_steps = int(batch_object_steps)
+    if round_steps is not None:
+        o.round_steps = int(round_steps)
+    o.outputs_on_device = int(bool(outputs_on_device))
+    o.inputs_on_device = int(bool(inputs_on_device))
+    return o
+
+
+def _mode(mode):
+    if isinstance(mode, str):
+        return {"grid": CD_GRID, "hybrid": CD_HYBRID}[mode]
+    return int(mode)
+
+
+def _torch_stream():
+    try:
+        import torch
+        if torch.cuda.is_available():
+            return torch.cuda.current_stream().cuda_stream
+    except Exception:
+        pass
+    return None
+
+
+def screen(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
+    """Conjunctions as a structured numpy array (CONJ_DTYPE), sorted by (i, j, step)."""
+    E = _Elements(pop)
+    st = cd_stats()
+    opt = make_options(inputs_on_device=E.on_device, **kw)
+    if opt.stream is None and E.on_device:
+        opt.stream = _torch_stream()
+    opt.stats = C.pointer(st)
+    out = cd_conjunctions()
+    _check(cd_screen_ex(E.s, E.n, float(t0), float(t1), float(dt), float(d), _mode(mode), opt, out))
+    try:
+        if opt.outputs_on_device:
+            raise ValueError("use screen_device() for device outputs")
+        if out.count:
+            buf = (C.c_char * (out.count * CONJ_DTYPE.itemsize)).from_address(out.data)
+            res = np.frombuffer(buf, dtype=CONJ_DTYPE).copy()
+        else:
+            res = np.zeros(0, dtype=CONJ_DTYPE)
+    finally:
+        cd_conjunctions_free(out)
+    return (res, st.as_dict()) if return_stats else res
+
+
+def candidates(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
+    """The level-1 candidate set K as a structured numpy array (CAND_DTYPE), sorted."""
+    E = _Elements(pop)
+    st = cd_stats()
+    opt = make_options(inputs_on_device=E.on_device, **kw)
+    opt.stats = C.pointer(st)
+    p = C.c_void_p()
+    cnt = C.c_size_t()
+    _check(cd_candidates(E.s, E.n, float(t0), float(t1), float(dt), float(d), _mode(mode), opt, p,
+                         cnt))
+    try:
+        if cnt.value:
+            buf = (C.c_char * (cnt.value * CAND_DTYPE.itemsize)).from_address(p.value)
+            res = np.frombuffer(buf, dtype=CAND_DTYPE).copy()
+        else:
+            res = np.zeros(0, dtype=CAND_DTYPE)
+    finally:
+        cd_candidates_free(p)
+    return (res, st.as_dict()) if return_stats else res
+
+
+def propagate(pop, times, velocity=False, **kw):
+    """Positions (nt, n, 3) [km] (and velocities [km/s]) at `times` [s from epoch]."""
+    E = _Elements(pop)
+    t = np.ascontiguousarray(np.atleast_1d(np.asarray(times, dtype=np.float64)))
+    xyz = np.zeros((t.size, E.n, 3))
+    v = np.zeros((t.size, E.n, 3)) if velocity else None
+    opt = make_options(inputs_on_device=E.on_device, **kw)
+    _check(cd_propagate(E.s, E.n, t.ctypes.data, t.size, xyz.ctypes.data,
+                        v.ctypes.data if velocity else None, opt))
+    return (xyz, v) if velocity else xyz
+

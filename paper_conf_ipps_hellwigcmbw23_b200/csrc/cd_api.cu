@@ -1,0 +1,652 @@
+// cd_api.cu -- C ABI (include/cdscreen.h) and host orchestration of the screening path.
+//
+// Structure of one call ("four major steps"):
+//   1) memory allocation (stream-ordered, pooled)
+//   2) per step batch: propagate + insert into the per-step hash grid, neighbour scan P:71
+//   3) (hybrid) orbital filter chain
+//   4) TCA/PCA refinement
+// The sampling steps are processed in rounds (bounded candidate queue, overflow -> retry) and
+// within a round in batches of B steps whose grids are in flight together (the paper's p
+// parallel grids).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/cdscreen.h"
+#include "cd_internal.h"
+#include "cd_hybrid.h"
+
+using namespace cdk;
+using namespace cdh;
+
+namespace {
+
+thread_local std::string g_err;
+
+cd_status fail(cd_status s, const char* fmt, ...)
+{
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return s;
+}
+
+#define CU(x)                                                                                   \
+    do {                                                                                        \
+        cudaError_t _e = (x);                                                                   \
+        if (_e != cudaSuccess)                                                                  \
+            return fail(_e == cudaErrorMemoryAllocation ? CD_ENOMEM : CD_ECUDA, "%s: %s (%s:%d)", \
+                        #x, cudaGetErrorString(_e), __FILE__, __LINE__);                         \
+    } while (0)
+
+#define TRY(x)                          \
+    do {                                \
+        cd_status _s = (x);             \
+        if (_s != CD_OK) return _s;     \
+    } while (0)
+
+// stream-ordered device buffer
+template <typename T>
+struct DBuf {
+    T* p = nullptr;
+    size_t n = 0;
+    cudaStream_t st = nullptr;
+    DBuf() = default;
+    explicit DBuf(cudaStream_t s) : st(s) {}
+    DBuf(const DBuf&) = delete;
+    DBuf& operator=(const DBuf&) = delete;
+    ~DBuf() { release(); }
+    void release()
+    {
+        if (p) cudaFreeAsync(p, st);
+        p = nullptr;
+        n = 0;
+    }
+    cudaError_t alloc(size_t count)
+    {
+        release();
+        n = count;
+        return cudaMallocAsync((void**)&p, sizeof(T) * (count ? count : 1), st);
+    }
+    T* detach()
+    {
+        T* q = p;
+        p = nullptr;
+        n = 0;
+        return q;
+    }
+};
+
+std::mutex g_pool_mu;
+bool g_pool_done[64] = {};
+
+void setup_pool(int dev)
+{
+    std::lock_guard<std::mutex> lk(g_pool_mu);
+    if (dev < 0 || dev >= 64 || g_pool_done[dev]) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = ~uint64_t(0);
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    g_pool_done[dev] = true;
+}
+
+struct Owner {
+    bool device;
+    void* p;
+};
+
+// One library call: device, stream, events, launch count.
+struct Call {
+    int prev_dev = -1, dev = -1;
+    cudaStream_t st = nullptr;
+    bool own_stream = false;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    LaunchCount lc;
+    ~Call()
+    {
+        if (ev0) cudaEventDestroy(ev0);
+        if (ev1) cudaEventDestroy(ev1);
+        if (own_stream && st) {
+            cudaStreamSynchronize(st);
+            cudaStreamDestroy(st);
+        }
+        if (prev_dev >= 0 && prev_dev != dev) cudaSetDevice(prev_dev);
+    }
+    cd_status begin(const cd_options& o)
+    {
+        int ndev = 0;
+        if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+            return fail(CD_ENODEV, "no CUDA device available");
+        CU(cudaGetDevice(&prev_dev));
+        dev = o.device >= 0 ? o.device : prev_dev;
+        if (dev >= ndev) return fail(CD_EINVAL, "device %d out of range (%d devices)", dev, ndev);
+        CU(cudaSetDevice(dev));
+        cudaDeviceProp prop;
+        CU(cudaGetDeviceProperties(&prop, dev));
+        if (prop.major != 10 || prop.minor != 0)
+            return fail(CD_ENODEV, "libcdscreen is built for sm_100a (B200); device %d is sm_%d%d",
+                        dev, prop.major, prop.minor);
+        setup_pool(dev);
+        if (o.stream) {
+            st = (cudaStream_t)o.stream;
+        } else {
+            CU(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+            own_stream = true;
+        }
+        CU(cudaEventCreate(&ev0));
+        CU(cudaEventCreate(&ev1));
+        CU(cudaEventRecord(ev0, st));
+        return CD_OK;
+    }
+};
+
+bool is_fin(double x) { return std::isfinite(x); }
+
+cd_status validate_scalars(size_t n, double t0, double t1, double dt, double d, const cd_options& o,
+                           int64_t* K)
+{
+    if (n >= 0xffffffffull) return fail(CD_EINVAL, "n = %zu must be < 2^32 - 1", n);
+    if (!is_fin(t0) || !is_fin(t1) || !(t1 >= t0)) return fail(CD_EINVAL, "need finite t1 >= t0");
+    if (!is_fin(dt) || !(dt > 0.0)) return fail(CD_EINVAL, "need dt > 0");
+    if (!is_fin(d) || !(d > 0.0)) return fail(CD_EINVAL, "need threshold d > 0");
+    if (!is_fin(o.v_margin) || o.v_margin < 0.0) return fail(CD_EINVAL, "need v_margin >= 0");
+    if (!(o.cell_factor >= 1.0) || !is_fin(o.cell_factor)) return fail(CD_EINVAL, "need cell_factor >= 1");
+    if (o.n_ranks < 1 || o.rank < 0 || o.rank >= o.n_ranks)
+        return fail(CD_EINVAL, "need 0 <= rank < n_ranks");
+    for (int c = 0; c < 3; ++c)
+        if (!is_fin(o.grid_origin[c])) return fail(CD_EINVAL, "grid_origin must be finite");
+    const double kk = std::floor((t1 - t0) / dt) + 1.0;
+    if (!(kk < 4294967295.0)) return fail(CD_EINVAL, "too many steps: K = %.0f", kk);
+    *K = (int64_t)kk;
+    return CD_OK;
+}
+
+// Validate element values (host copy) -- a > 0, 0 <= e < 1, finite angles.
+cd_status validate_elements_host(const double* const v[6], size_t n)
+{
+    for (size_t i = 0; i < n; ++i) {
+        const double a = v[0][i], e = v[1][i];
+        if (!(a > 0.0) || !is_fin(a)) return fail(CD_EINVAL, "element %zu: a = %g must be > 0", i, a);
+        if (!(e >= 0.0 && e < 1.0)) return fail(CD_EINVAL, "element %zu: e = %g must be in [0, 1)", i, e);
+        for (int c = 2; c < 6; ++c)
+            if (!is_fin(v[c][i])) return fail(CD_EINVAL, "element %zu: non-finite angle", i);
+    }
+    return CD_OK;
+}
+
+__global__ void k_validate(Elements el, int64_t n, int* bad)
+{
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const double a = el.a[i], e = el.e[i];
+    bool ok = a > 0.0 && isfinite(a) && e >= 0.0 && e < 1.0 && isfinite(el.inc[i]) &&
+              isfinite(el.raan[i]) && isfinite(el.argp[i]) && isfinite(el.nu0[i]);
+    if (!ok) atomicMin(bad, (int)(i < 0x7fffffff ? i : 0x7ffffffe));
+}
+
+// Device-resident orbit records of one call (internal order sorted by eccentricity class).
+struct OrbitSet {
+    DBuf<double> rec;
+    DBuf<uint8_t> cls;
+    DBuf<uint32_t> perm;   // internal -> caller index
+    Orbits view() const
+    {
+        Orbits O;
+        O.rec = rec.p;
+        O.cls = cls.p;
+        O.n = (int64_t)perm.n;
+        return O;
+    }
+};
+
+cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_options& o, OrbitSet& S)
+{
+    if (!el || !el->a || !el->e || !el->inc || !el->raan || !el->argp || !el->nu0)
+        return fail(CD_EINVAL, "elements must be non-NULL");
+    cudaStream_t st = C.st;
+    S.rec.st = S.cls.st = S.perm.st = st;
+    DBuf<double> up(st);
+    Elements E;
+    const double* src[6] = {el->a, el->e, el->inc, el->raan, el->argp, el->nu0};
+    if (o.inputs_on_device) {
+        E = Elements{el->a, el->e, el->inc, el->raan, el->argp, el->nu0};
+        DBuf<int> bad(st);
+        CU(bad.alloc(1));
+        int init = 0x7fffffff;
+        CU(cudaMemcpyAsync(bad.p, &init, sizeof(int), cudaMemcpyHostToDevice, st));
+        k_validate<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(E, (int64_t)n, bad.p);
+        C.lc.bump();
+        CU(cudaGetLastError());
+        int hb = 0;
+        CU(cudaMemcpyAsync(&hb, bad.p, sizeof(int), cudaMemcpyDeviceToHost, st));
+        CU(cudaStreamSynchronize(st));
+        if (hb != 0x7fffffff) return fail(CD_EINVAL, "element %d: invalid (need a > 0, 0 <= e < 1, finite)", hb);
+    } else {
+        TRY(validate_elements_host(src, n));
+        CU(up.alloc(6 * n));
+        for (int c = 0; c < 6; ++c)
+            CU(cudaMemcpyAsync(up.p + c * n, src[c], sizeof(double) * n, cudaMemcpyHostToDevice, st));
+        E = Elements{up.p, up.p + n, up.p + 2 * n, up.p + 3 * n, up.p + 4 * n, up.p + 5 * n};
+    }
+    DBuf<uint32_t> key(st), idx(st), keyo(st);
+    CU(key.alloc(n));
+    CU(idx.alloc(n));
+    CU(keyo.alloc(n));
+    CU(S.perm.alloc(n));
+    CU(launch_classify(E, (int64_t)n, key.p, idx.p, st, C.lc));
+    CU(sort_pairs_u32(key.p, keyo.p, idx.p, S.perm.p, n, 3, st, C.lc));
+    CU(S.rec.alloc((size_t)kNCol * n));
+    CU(S.cls.alloc(n));
+    CU(launch_build_records(E, S.perm.p, (int64_t)n, S.rec.p, S.cls.p, st, C.lc));
+    return CD_OK;
+}
+
+uint64_t next_pow2(uint64_t x)
+{
+    uint64_t p = 1;
+    while (p < x) p <<= 1;
+    return p;
+}
+
+enum class Want { Conj, Cand };
+
+struct Result {
+    DBuf<Conj> conj;        // unsorted conjunction records (internal ids)
+    size_t n_conj = 0;
+    DBuf<Cand> cand;        // accumulated candidates (cd_candidates)
+    size_t n_cand = 0;
+};
+
+// The screening loop over this rank's step slice.
+cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, double d, cd_mode mode,
+              const cd_options& o, int64_t K, Want want, Result& R, cd_stats& stats)
+{
+    cudaStream_t st = C.st;
+    const Orbits O = S.view();
+    const int64_t n = O.n;
+    const int64_t kb = (int64_t)((__int128)K * o.rank / o.n_ranks);
+    const int64_t ke = (int64_t)((__int128)K * (o.rank + 1) / o.n_ranks);
+    stats.steps = (uint64_t)(ke - kb);
+    stats.object_steps = (uint64_t)(ke - kb) * (uint64_t)n;
+    const double gc = d + o.v_margin * dt;   // Eq. 1
+    double L = gc * o.cell_factor;
+    if (L < gc * (1.0 + 1e-12)) L = gc * (1.0 + 1e-12);
+    GridGeom g;
+    g.ox = o.grid_origin[0];
+    g.oy = o.grid_origin[1];
+    g.oz = o.grid_origin[2];
+    g.inv_cell = 1.0 / L;
+    g.gc2 = gc * gc;
+    RefineParams P{t0, t1, dt, d, gc};
+
+    R.conj.st = R.cand.st = st;
+    if (ke <= kb || n < 2) return CD_OK;
+
+    const uint64_t M = next_pow2((uint64_t)std::max<int64_t>(2 * n, 64));   // 2n slots
+    const uint64_t mask = M - 1;
+    const size_t target = o.batch_object_steps ? o.batch_object_steps : (size_t(1) << 20);
+    int64_t Bmax = std::max<int64_t>(1, (int64_t)(target / (size_t)n));
+    Bmax = std::min<int64_t>(Bmax, std::min<int64_t>(ke - kb, 65535));
+
+    DBuf<Slot> tabs(st);
+    DBuf<Entry> ents(st);
+    CU(tabs.alloc((size_t)Bmax * M));
+    CU(ents.alloc((size_t)Bmax * n));
+    size_t qcap = std::max<size_t>(size_t(1) << 22, 4 * (size_t)n);
+    DBuf<Cand> q(st);
+    CU(q.alloc(qcap));
+    size_t wcap = want == Want::Conj ? qcap : 0;
+    DBuf<Work> w(st);
+    if (want == Want::Conj) CU(w.alloc(wcap));
+    size_t ocap = size_t(1) << 20;
+    if (want == Want::Conj) CU(R.conj.alloc(ocap));
+    size_t ccap = want == Want::Cand ? (size_t(1) << 20) : 0;
+    if (want == Want::Cand) CU(R.cand.alloc(ccap));
+
+    DBuf<Ctrl> ctrl(st);
+    CU(ctrl.alloc(1));
+    CU(cudaMemsetAsync(ctrl.p, 0, sizeof(Ctrl), st));
+    DBuf<unsigned long long> nwork(st);
+    CU(nwork.alloc(1));
+    Ctrl* hctrl = nullptr;
+    CU(cudaMallocHost((void**)&hctrl, sizeof(Ctrl) + sizeof(unsigned long long)));
+    struct HostFree {
+        void* p;
+        ~HostFree() { cudaFreeHost(p); }
+    } hf{hctrl};
+    unsigned long long* hnwork = reinterpret_cast<unsigned long long*>(hctrl + 1);
+
+    int64_t Rsteps = o.round_steps ? (int64_t)o.round_steps
+                                   : std::max<int64_t>(1, (int64_t)(qcap / 2 / (size_t)std::max<int64_t>(1, n / 20)));
+    unsigned long long conj_before = 0;
+    int64_t k = kb;
+    while (k < ke) {
+        const int64_t Rk = std::min<int64_t>(Rsteps, ke - k);
+        CU(cudaMemsetAsync(&ctrl.p->n_cand, 0, sizeof(unsigned long long), st));
+        CU(cudaMemsetAsync(nwork.p, 0, sizeof(unsigned long long), st));
+        for (int64_t kk = k; kk < k + Rk; kk += Bmax) {
+            const int B = (int)std::min<int64_t>(Bmax, k + Rk - kk);
+            CU(launch_fill_u64(reinterpret_cast<unsigned long long*>(tabs.p), (size_t)B * M * 2,
+                               ~0ull, st, C.lc));
+            CU(launch_prop_insert(O, g, tabs.p, ents.p, mask, kk, B, t0, dt, ctrl.p, st, C.lc));
+            CU(launch_scan(g, tabs.p, ents.p, n, mask, kk, B, q.p, qcap, ctrl.p, st, C.lc));
+        }
+        if (want == Want::Conj) {
+            if (mode == CD_HYBRID) {
+                CU(launch_hybrid_filter(O, P, q.p, qcap, w.p, wcap, nwork.p, R.conj.p, ocap, ctrl.p,
+                                        st, C.lc));
+                CU(launch_hybrid_brent(O, P, w.p, nwork.p, wcap, R.conj.p, ocap, ctrl.p, st, C.lc));
+            } else {
+                CU(launch_prefilter(O, P, q.p, qcap, w.p, wcap, nwork.p, R.conj.p, ocap, ctrl.p, st,
+                                    C.lc));
+                CU(launch_brent(O, P, w.p, nwork.p, wcap, R.conj.p, ocap, ctrl.p, st, C.lc));
+            }
+        }
+        CU(cudaMemcpyAsync(hctrl, ctrl.p, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
+        CU(cudaMemcpyAsync(hnwork, nwork.p, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+        CU(cudaStreamSynchronize(st));
+        if (hctrl->err_range)
+            return fail(CD_ERANGE, "a position fell outside the cell-key range (+-%lld cells of %g km)",
+                        (long long)kCellMax, L);
+        bool redo = false;
+        if (hctrl->n_cand > qcap) {
+            ++stats.retries;
+            if (Rk > 1) {
+                const double rate = (double)hctrl->n_cand / (double)Rk;
+                Rsteps = std::max<int64_t>(1, std::min<int64_t>(Rk / 2, (int64_t)(0.5 * qcap / rate)));
+            } else {
+                qcap = (size_t)(hctrl->n_cand * 1.25) + 1024;
+                CU(q.alloc(qcap));
+                if (want == Want::Conj) {
+                    wcap = qcap;
+                    CU(w.alloc(wcap));
+                }
+            }
+            redo = true;
+        } else if (want == Want::Conj && *hnwork > wcap) {
+            ++stats.retries;
+            wcap = (size_t)(*hnwork * 1.25) + 1024;
+            CU(w.alloc(wcap));
+            redo = true;
+        } else if (want == Want::Conj && hctrl->n_conj > ocap) {
+            ++stats.retries;
+            const size_t ncap = std::max<size_t>(2 * ocap, (size_t)(hctrl->n_conj * 1.25) + 1024);
+            DBuf<Conj> nb(st);
+            CU(nb.alloc(ncap));
+            if (conj_before)
+                CU(cudaMemcpyAsync(nb.p, R.conj.p, sizeof(Conj) * conj_before, cudaMemcpyDeviceToDevice, st));
+            std::swap(R.conj.p, nb.p);
+            std::swap(R.conj.n, nb.n);
+            ocap = ncap;
+            redo = true;
+        }
+        if (redo) {
+            CU(cudaMemcpyAsync(&ctrl.p->n_conj, &conj_before, sizeof(unsigned long long),
+                               cudaMemcpyHostToDevice, st));
+            CU(cudaStreamSynchronize(st));
+            continue;
+        }
+        // round accepted
+        stats.candidates += hctrl->n_cand;
+        stats.refined += *hnwork;
+        if (want == Want::Cand && hctrl->n_cand) {
+            if (R.n_cand + hctrl->n_cand > ccap) {
+                const size_t ncap = std::max<size_t>(2 * ccap, R.n_cand + hctrl->n_cand + 1024);
+                DBuf<Cand> nb(st);
+                CU(nb.alloc(ncap));
+                if (R.n_cand)
+                    CU(cudaMemcpyAsync(nb.p, R.cand.p, sizeof(Cand) * R.n_cand, cudaMemcpyDeviceToDevice, st));
+                std::swap(R.cand.p, nb.p);
+                std::swap(R.cand.n, nb.n);
+                ccap = ncap;
+            }
+            CU(cudaMemcpyAsync(R.cand.p + R.n_cand, q.p, sizeof(Cand) * hctrl->n_cand,
+                               cudaMemcpyDeviceToDevice, st));
+            R.n_cand += hctrl->n_cand;
+        }
+        conj_before = hctrl->n_conj;
+        if (!o.round_steps) {
+            const double rate = std::max(1.0, (double)hctrl->n_cand / (double)Rk);
+            Rsteps = std::max<int64_t>(1, std::min<int64_t>(1 << 16, (int64_t)(0.5 * qcap / rate)));
+        }
+        k += Rk;
+    }
+    R.n_conj = (size_t)conj_before;
+    stats.hybrid_ap_rejected = hctrl->n_ap;
+    stats.hybrid_coplanar = hctrl->n_coplanar;
+    stats.hybrid_path_rejected = hctrl->n_path;
+    stats.hybrid_time_rejected = hctrl->n_time;
+    return CD_OK;
+}
+
+cd_options defaults()
+{
+    cd_options o;
+    cd_options_init(&o);
+    return o;
+}
+
+cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,
+                      cd_mode mode, const cd_options* opt, cd_conjunctions* out)
+{
+    if (!out) return fail(CD_EINVAL, "out must be non-NULL");
+    out->data = nullptr;
+    out->count = 0;
+    out->_owner = nullptr;
+    const cd_options o = opt ? *opt : defaults();
+    if (mode != CD_GRID && mode != CD_HYBRID) return fail(CD_EINVAL, "unknown mode %d", (int)mode);
+    int64_t K = 0;
+    TRY(validate_scalars(n, t0, t1, dt, d, o, &K));
+    cd_stats stats;
+    memset(&stats, 0, sizeof stats);
+    Call C;
+    TRY(C.begin(o));
+    Result R;
+    DBuf<Conj> sorted(C.st);
+    {
+        OrbitSet S;
+        if (n > 0) TRY(prepare_orbits(C, el, n, o, S));
+        else if (!el) return fail(CD_EINVAL, "elements must be non-NULL");
+        TRY(run(C, S, t0, t1, dt, d, mode, o, K, Want::Conj, R, stats));
+        if (R.n_conj) {
+            CU(sorted.alloc(R.n_conj));
+            CU(finalize_conj(R.conj.p, R.n_conj, S.perm.p, sorted.p, C.st, C.lc));
+        }
+    }
+    Owner* own = new Owner{o.outputs_on_device != 0, nullptr};
+    if (R.n_conj) {
+        if (o.outputs_on_device) {
+            own->p = sorted.detach();
+        } else {
+            void* h = malloc(sizeof(cd_conjunction) * R.n_conj);
+            if (!h) {
+                delete own;
+                return fail(CD_ENOMEM, "host allocation of %zu records failed", R.n_conj);
+            }
+            CU(cudaMemcpyAsync(h, sorted.p, sizeof(cd_conjunction) * R.n_conj, cudaMemcpyDeviceToHost, C.st));
+            own->p = h;
+        }
+    }
+    CU(cudaEventRecord(C.ev1, C.st));
+    CU(cudaEventSynchronize(C.ev1));
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, C.ev0, C.ev1);
+    stats.ms_total = ms;
+    stats.conjunctions = R.n_conj;
+    stats.kernel_launches = C.lc.n;
+    if (o.stats) *o.stats = stats;
+    out->data = static_cast<cd_conjunction*>(own->p);
+    out->count = R.n_conj;
+    out->_owner = own;
+    return CD_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+void cd_options_init(cd_options* o)
+{
+    if (!o) return;
+    memset(o, 0, sizeof *o);
+    o->v_margin = 7.8;   // Eq. 1: typical LEO speed
+    o->device = -1;
+    o->rank = 0;
+    o->n_ranks = 1;
+    o->cell_factor = 1.0;
+}
+
+cd_status cd_screen(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,
+                    cd_mode mode, cd_conjunctions* out)
+{
+    return cd_screen_ex(el, n, t0, t1, dt, d, mode, nullptr, out);
+}
+
+cd_status cd_screen_ex(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,
+                       cd_mode mode, const cd_options* opt, cd_conjunctions* out)
+{
+    try {
+        return screen_impl(el, n, t0, t1, dt, d, mode, opt, out);
+    } catch (...) {
+        return fail(CD_EINTERNAL, "unexpected C++ exception");
+    }
+}
+
+cd_status cd_candidates(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,
+                        cd_mode mode, const cd_options* opt, cd_candidate** out, size_t* count)
+{
+    try {
+        if (!out || !count) return fail(CD_EINVAL, "out and count must be non-NULL");
+        *out = nullptr;
+        *count = 0;
+        if (mode != CD_GRID && mode != CD_HYBRID) return fail(CD_EINVAL, "unknown mode %d", (int)mode);
+        const cd_options o = opt ? *opt : defaults();
+        int64_t K = 0;
+        TRY(validate_scalars(n, t0, t1, dt, d, o, &K));
+        cd_stats stats;
+        memset(&stats, 0, sizeof stats);
+        Call C;
+        TRY(C.begin(o));
+        Result R;
+        DBuf<Cand> sorted(C.st);
+        OrbitSet S;
+        if (n > 0) TRY(prepare_orbits(C, el, n, o, S));
+        TRY(run(C, S, t0, t1, dt, d, mode, o, K, Want::Cand, R, stats));
+        cd_candidate* h = nullptr;
+        if (R.n_cand) {
+            CU(sorted.alloc(R.n_cand));
+            CU(finalize_cand(R.cand.p, R.n_cand, S.perm.p, sorted.p, C.st, C.lc));
+            h = (cd_candidate*)malloc(sizeof(cd_candidate) * R.n_cand);
+            if (!h) return fail(CD_ENOMEM, "host allocation failed");
+            cudaError_t e = cudaMemcpyAsync(h, sorted.p, sizeof(cd_candidate) * R.n_cand,
+                                            cudaMemcpyDeviceToHost, C.st);
+            if (e == cudaSuccess) e = cudaStreamSynchronize(C.st);
+            if (e != cudaSuccess) {
+                free(h);
+                return fail(CD_ECUDA, "copy-out: %s", cudaGetErrorString(e));
+            }
+        }
+        CU(cudaEventRecord(C.ev1, C.st));
+        CU(cudaEventSynchronize(C.ev1));
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, C.ev0, C.ev1);
+        stats.ms_total = ms;
+        stats.kernel_launches = C.lc.n;
+        if (o.stats) *o.stats = stats;
+        *out = h;
+        *count = R.n_cand;
+        return CD_OK;
+    } catch (...) {
+        return fail(CD_EINTERNAL, "unexpected C++ exception");
+    }
+}
+
+cd_status cd_propagate(const cd_elements* el, size_t n, const double* t, size_t nt, double* xyz,
+                       double* vxyz, const cd_options* opt)
+{
+    try {
+        if (!xyz || (!t && nt)) return fail(CD_EINVAL, "t and xyz must be non-NULL");
+        if (n == 0 || nt == 0) return CD_OK;
+        if (n >= 0xffffffffull) return fail(CD_EINVAL, "n too large");
+        for (size_t q = 0; q < nt; ++q)
+            if (!is_fin(t[q])) return fail(CD_EINVAL, "non-finite time");
+        const cd_options o = opt ? *opt : defaults();
+        Call C;
+        TRY(C.begin(o));
+        OrbitSet S;
+        TRY(prepare_orbits(C, el, n, o, S));
+        DBuf<double> dt_(C.st), dx(C.st), dv(C.st);
+        CU(dt_.alloc(nt));
+        CU(dx.alloc(nt * n * 3));
+        if (vxyz) CU(dv.alloc(nt * n * 3));
+        CU(cudaMemcpyAsync(dt_.p, t, sizeof(double) * nt, cudaMemcpyHostToDevice, C.st));
+        CU(launch_propagate_out(S.view(), S.perm.p, dt_.p, (int64_t)nt, dx.p, vxyz ? dv.p : nullptr,
+                                C.st, C.lc));
+        CU(cudaMemcpyAsync(xyz, dx.p, sizeof(double) * nt * n * 3, cudaMemcpyDeviceToHost, C.st));
+        if (vxyz) CU(cudaMemcpyAsync(vxyz, dv.p, sizeof(double) * nt * n * 3, cudaMemcpyDeviceToHost, C.st));
+        CU(cudaStreamSynchronize(C.st));
+        if (o.stats) {
+            cd_stats s;
+            memset(&s, 0, sizeof s);
+            s.kernel_launches = C.lc.n;
+            *o.stats = s;
+        }
+        return CD_OK;
+    } catch (...) {
+        return fail(CD_EINTERNAL, "unexpected C++ exception");
+    }
+}
+
+void cd_conjunctions_free(cd_conjunctions* c)
+{
+    if (!c) return;
+    Owner* own = static_cast<Owner*>(c->_owner);
+    if (own) {
+        if (own->p) {
+            if (own->device) cudaFree(own->p);
+            else free(own->p);
+        }
+        delete own;
+    }
+    c->data = nullptr;
+    c->count = 0;
+    c->_owner = nullptr;
+}
+
+void cd_candidates_free(cd_candidate* c) { free(c); }
+
+const char* cd_status_str(cd_status s)
+{
+    switch (s) {
+    case CD_OK: return "CD_OK";
+    case CD_EINVAL: return "CD_EINVAL";
+    case CD_ENOMEM: return "CD_ENOMEM";
+    case CD_ECUDA: return "CD_ECUDA";
+    case CD_ENCCL: return "CD_ENCCL";
+    case CD_ERANGE: return "CD_ERANGE";
+    case CD_EINTERNAL: return "CD_EINTERNAL";
+    case CD_ENODEV: return "CD_ENODEV";
+    }
+    return "CD_UNKNOWN";
+}
+
+const char* cd_last_error(void) { return g_err.c_str(); }
+
+int cd_abi_version(void) { return CD_ABI_VERSION; }
+
+uint64_t cd_kernel_launches(void) { return cdh::g_launches.load(); }
+
+}  // extern "C"

@@ -1,0 +1,442 @@
+// cd_kernels.cu -- CUDA kernels of the screening hot path (sm_100a, fp64, no tensor cores).
+//
+//   a1 precompute     k_classify, k_build_records   ("precalculating the reusable
+//                                                     parts ... once", P:236 a_k)
+//   a2-a4 propagate + cell key + hash insert        k_prop_insert  (Eq. 2)
+//   a5-a6 27-cell neighbour scan + candidate queue  k_scan
+//   a7 refinement     k_prefilter (conservative linear bound), k_brent
+#include <cooperative_groups.h>
+
+#include "cd_internal.h"
+
+namespace cg = cooperative_groups;
+using namespace cdk;
+
+namespace cdh {
+
+std::atomic<uint64_t> g_launches{0};
+
+static inline unsigned blocks_for(int64_t n, int t) { return (unsigned)((n + t - 1) / t); }
+
+// Warp-aggregated append: one atomicAdd per group of converged lanes.  The counter keeps
+// counting past `cap` so the host can detect overflow and size the retry.
+template <typename T>
+__device__ __forceinline__ void append(T* buf, size_t cap, unsigned long long* cnt, const T& v)
+{
+    cg::coalesced_group g = cg::coalesced_threads();
+    unsigned long long base = 0;
+    if (g.thread_rank() == 0) base = atomicAdd(cnt, (unsigned long long)g.size());
+    base = g.shfl(base, 0);
+    const unsigned long long idx = base + g.thread_rank();
+    if (idx < cap) buf[idx] = v;
+}
+
+// ---------------------------------------------------------------------------------------
+// a1: per-object precompute
+// ---------------------------------------------------------------------------------------
+__global__ void k_classify(Elements el, int64_t n, uint32_t* key, uint32_t* idx)
+{
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    key[i] = (uint32_t)ecc_class(el.e[i]);
+    idx[i] = (uint32_t)i;
+}
+
+__global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, int64_t n,
+                                double* __restrict__ rec, uint8_t* __restrict__ cls)
+{
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (r >= n) return;
+    const uint32_t i = perm[r];
+    const double a = el.a[i], e = el.e[i], inc = el.inc[i];
+    const double raan = el.raan[i], argp = el.argp[i], nu0 = el.nu0[i];
+    double sO, cO, sw, cw, si, ci;
+    sincos(raan, &sO, &cO);
+    sincos(argp, &sw, &cw);
+    sincos(inc, &si, &ci);
+    // perifocal unit vectors (Fig. 8: rotation by Omega, i, omega)
+    const double P[3] = {cO * cw - sO * sw * ci, sO * cw + cO * sw * ci, sw * si};
+    const double Q[3] = {-cO * sw - sO * cw * ci, -sO * sw + cO * cw * ci, cw * si};
+    const double b = a * sqrt((1.0 - e) * (1.0 + e));
+    // true anomaly at epoch -> eccentric -> mean anomaly
+    double sh, ch;
+    sincos(0.5 * nu0, &sh, &ch);
+    const double E0 = 2.0 * atan2(sqrt(1.0 - e) * sh, sqrt(1.0 + e) * ch);
+    const double M0 = E0 - e * sin(E0);
+    auto put = [&](int c, double v) { rec[c * n + r] = v; };
+    put(kM0, M0);
+    put(kNm, sqrt(kMu / (a * a * a)));
+    put(kE, e);
+    put(kAPx, a * P[0]); put(kAPy, a * P[1]); put(kAPz, a * P[2]);
+    put(kBQx, b * Q[0]); put(kBQy, b * Q[1]); put(kBQz, b * Q[2]);
+    put(kQper, a * (1.0 - e));
+    const double rho = 0.5 * e;
+    put(kEcr, e * cos(rho));
+    put(kEsr, e * sin(rho));
+    const int cl = ecc_class(e);
+    const int N = class_points(cl);
+    for (int j = 1; j <= (N - 2) / 2; ++j) {
+        const double ct = kNodes[cl][j - 1][0], st = kNodes[cl][j - 1][1];
+        put(kTab + 4 * (j - 1) + 0, e * cos(rho * ct));
+        put(kTab + 4 * (j - 1) + 1, e * sin(rho * ct));
+        put(kTab + 4 * (j - 1) + 2, cosh(rho * st));
+        put(kTab + 4 * (j - 1) + 3, sinh(rho * st));
+    }
+    cls[r] = (uint8_t)cl;
+}
+
+__global__ void k_propagate_out(Orbits O, const uint32_t* __restrict__ perm,
+                                const double* __restrict__ t, int64_t nt, double* xyz, double* vxyz)
+{
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t q = blockIdx.y;
+    if (r >= O.n || q >= nt) return;
+    double p[3], v[3];
+    const int64_t o = (q * O.n + perm[r]) * 3;
+    if (vxyz) {
+        state<true>(O, r, t[q], p, v);
+        vxyz[o] = v[0]; vxyz[o + 1] = v[1]; vxyz[o + 2] = v[2];
+    } else {
+        state<false>(O, r, t[q], p, v);
+    }
+    xyz[o] = p[0]; xyz[o + 1] = p[1]; xyz[o + 2] = p[2];
+}
+
+cudaError_t launch_classify(const Elements& el, int64_t n, uint32_t* key, uint32_t* idx,
+                            cudaStream_t st, LaunchCount& lc)
+{
+    k_classify<<<blocks_for(n, 256), 256, 0, st>>>(el, n, key, idx);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_build_records(const Elements& el, const uint32_t* perm, int64_t n, double* rec,
+                                 uint8_t* cls, cudaStream_t st, LaunchCount& lc)
+{
+    k_build_records<<<blocks_for(n, 128), 128, 0, st>>>(el, perm, n, rec, cls);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_propagate_out(const Orbits& O, const uint32_t* perm, const double* t, int64_t nt,
+                                 double* xyz, double* vxyz, cudaStream_t st, LaunchCount& lc)
+{
+    for (int64_t q0 = 0; q0 < nt; q0 += 65535) {
+        const int64_t m = nt - q0 < 65535 ? nt - q0 : 65535;
+        dim3 grid(blocks_for(O.n, 128), (unsigned)m);
+        k_propagate_out<<<grid, 128, 0, st>>>(O, perm, t + q0, m, xyz + q0 * O.n * 3,
+                                             vxyz ? vxyz + q0 * O.n * 3 : nullptr);
+        lc.bump();
+    }
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------------------
+// a4 helper: clear hash tables to the empty marker ("initialized with this value")
+// ---------------------------------------------------------------------------------------
+__global__ void k_fill_u64(ulonglong2* __restrict__ p, size_t n2, unsigned long long v)
+{
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n2; i += stride)
+        p[i] = make_ulonglong2(v, v);
+}
+
+cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long long v,
+                            cudaStream_t st, LaunchCount& lc)
+{
+    const size_t n2 = count / 2;   // count is even (slots are 2 words)
+    unsigned blocks = (unsigned)((n2 + 255) / 256);
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (blocks == 0) blocks = 1;
+    k_fill_u64<<<blocks, 256, 0, st>>>(reinterpret_cast<ulonglong2*>(p), n2, v);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------------------
+// a2-a4: one thread per (object, step): propagate (Contour), cell key, non-blocking insert.
+// Insertion: 64-bit CAS of the cell key into the first empty slot of its linear
+// probe sequence s_{i+1} = s_i + 1 mod M (Eq. 2); a slot already holding the same key is the
+// same cell, so the object is pushed onto that cell's singly linked list with an atomic
+// exchange of the list head (entries pre-allocated, one per object).
+// ---------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_prop_insert(Orbits O, GridGeom g, Slot* __restrict__ tabs,
+                                                     Entry* __restrict__ ents, uint64_t mask,
+                                                     int64_t k0, double t0, double dt, Ctrl* ctrl)
+{
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (r >= O.n) return;
+    const int s = blockIdx.y;
+    const double t = fma((double)(k0 + s), dt, t0);
+    double p[3], v[3];
+    state<false>(O, r, t, p, v);
+    int64_t c[3];
+    uint32_t prev = kNil;
+    if (cell_of(g, p, c)) {
+        Slot* tab = tabs + (size_t)s * (mask + 1);
+        const unsigned long long key = pack_key(c[0], c[1], c[2]);
+        uint64_t h = fmix64(key) & mask;
+        while (true) {
+            const unsigned long long old = atomicCAS(&tab[h].key, (unsigned long long)kEmpty, key);
+            if (old == kEmpty || old == key) break;
+            h = (h + 1) & mask;
+        }
+        prev = atomicExch(&tab[h].head, (uint32_t)r);
+    } else {
+        ctrl->err_range = 1;
+    }
+    Entry en;
+    en.x = p[0];
+    en.y = p[1];
+    en.z = p[2];
+    en.next = prev;
+    en.pad = 0;
+    ents[(size_t)s * O.n + r] = en;
+}
+
+cudaError_t launch_prop_insert(const Orbits& O, const GridGeom& g, Slot* tabs, Entry* ents,
+                               uint64_t mask, int64_t k0, int B, double t0, double dt, Ctrl* ctrl,
+                               cudaStream_t st, LaunchCount& lc)
+{
+    dim3 grid(blocks_for(O.n, 256), (unsigned)B);
+    k_prop_insert<<<grid, 256, 0, st>>>(O, g, tabs, ents, mask, k0, t0, dt, ctrl);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------------------
+// a5-a6: neighbour scan.  One thread per (object, step).  The object's own cell and the 13
+// cells of the positive half-shell are probed, which visits every unordered pair of cells in
+// a 3x3x3 neighbourhood exactly once ("every other satellite in that cell or the
+// 3^3-1 = 26 neighbor cells"; "prevent considering possible conjunctions twice").
+// A pair is a candidate iff |r_i - r_j| < g_c (reading R6); candidates are appended to the
+// queue with one atomic per group of converged lanes.
+// ---------------------------------------------------------------------------------------
+__constant__ int8_t kHalfShell[14][3] = {
+    {0, 0, 0},
+    {1, -1, -1}, {1, -1, 0}, {1, -1, 1}, {1, 0, -1}, {1, 0, 0}, {1, 0, 1}, {1, 1, -1}, {1, 1, 0}, {1, 1, 1},
+    {0, 1, -1}, {0, 1, 0}, {0, 1, 1},
+    {0, 0, 1}};
+
+__device__ __forceinline__ uint32_t probe(const Slot* __restrict__ tab, uint64_t mask,
+                                         unsigned long long key)
+{
+    uint64_t h = fmix64(key) & mask;
+    while (true) {
+        const ulonglong2 sl = __ldg(reinterpret_cast<const ulonglong2*>(tab + h));
+        if (sl.x == key) return (uint32_t)sl.y;
+        if (sl.x == kEmpty) return kNil;
+        h = (h + 1) & mask;
+    }
+}
+
+__global__ void __launch_bounds__(256) k_scan(GridGeom g, const Slot* __restrict__ tabs,
+                                              const Entry* __restrict__ ents, int64_t n, uint64_t mask,
+                                              int64_t k0, Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
+{
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (r >= n) return;
+    const int s = blockIdx.y;
+    const Slot* tab = tabs + (size_t)s * (mask + 1);
+    const Entry* E = ents + (size_t)s * n;
+    const Entry me = E[r];
+    const double p[3] = {me.x, me.y, me.z};
+    int64_t c[3];
+    if (!cell_of(g, p, c)) return;
+    const uint32_t step = (uint32_t)(k0 + s);
+#pragma unroll 1
+    for (int o = 0; o < 14; ++o) {
+        const unsigned long long key =
+            pack_key(c[0] + kHalfShell[o][0], c[1] + kHalfShell[o][1], c[2] + kHalfShell[o][2]);
+        uint32_t j = probe(tab, mask, key);
+        while (j != kNil) {
+            const Entry ej = E[j];
+            if (o != 0 || j > (uint32_t)r) {
+                const double dx = p[0] - ej.x, dy = p[1] - ej.y, dz = p[2] - ej.z;
+                if (fma(dx, dx, fma(dy, dy, dz * dz)) < g.gc2) {
+                    Cand cd;
+                    cd.i = (uint32_t)r < j ? (uint32_t)r : j;
+                    cd.j = (uint32_t)r < j ? j : (uint32_t)r;
+                    cd.step = step;
+                    append(q, qcap, &ctrl->n_cand, cd);
+                }
+            }
+            j = ej.next;
+        }
+    }
+}
+
+cudaError_t launch_scan(const GridGeom& g, const Slot* tabs, const Entry* ents, int64_t n,
+                        uint64_t mask, int64_t k0, int B, Cand* q, size_t qcap, Ctrl* ctrl,
+                        cudaStream_t st, LaunchCount& lc)
+{
+    dim3 grid(blocks_for(n, 256), (unsigned)B);
+    k_scan<<<grid, 256, 0, st>>>(g, tabs, ents, n, mask, k0, q, qcap, ctrl);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------------------
+// a7: refinement.
+// (1) k_prefilter: state of both objects at t_k.  Degenerate pairs (|dv| < 1e-9 km/s) are
+//     reported directly (tca = t_k).  Otherwise a conservative bound discards candidates that
+//     cannot have a local minimum below d in the owner cell [t_k - dt/2, t_k + dt/2]:
+//         D(t_k + tau) >= |dr + tau dv| - tau^2/2 * (mu/q_i^2 + mu/q_j^2)
+//     (Taylor remainder, |acceleration| <= mu / perigee^2).  Survivors become work items with
+//     the Brent half-window t_w = 2 g_c / min(|v_i|, |v_j|).
+// (2) k_brent: Brent's minimisation (golden section + parabolic interpolation, ref. [44],
+//     Boost's implementation in the paper) of D^2(t_k + tau) over
+//     tau in [-t_w, t_w] intersected with [t0, t1]; a minimum at an end of the interval is
+//     discarded ("the minimum will be found when considering the neighboring
+//     interval"); otherwise it is reported iff its owner step is k and D < d.
+// ---------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_prefilter(Orbits O, RefineParams P, const Cand* __restrict__ q,
+                                                   size_t qcap, Work* __restrict__ w, size_t wcap,
+                                                   unsigned long long* n_work, Conj* __restrict__ out,
+                                                   size_t ocap, Ctrl* ctrl)
+{
+    unsigned long long nc = ctrl->n_cand;
+    if (nc > qcap) nc = qcap;
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < nc; idx += stride) {
+        const Cand cd = q[idx];
+        const double tk = fma((double)cd.step, P.dt, P.t0);
+        double ri[3], vi[3], rj[3], vj[3];
+        state<true>(O, cd.i, tk, ri, vi);
+        state<true>(O, cd.j, tk, rj, vj);
+        const double dr[3] = {ri[0] - rj[0], ri[1] - rj[1], ri[2] - rj[2]};
+        const double dv[3] = {vi[0] - vj[0], vi[1] - vj[1], vi[2] - vj[2]};
+        const double dv2 = dv[0] * dv[0] + dv[1] * dv[1] + dv[2] * dv[2];
+        const double dr2 = dr[0] * dr[0] + dr[1] * dr[1] + dr[2] * dr[2];
+        if (sqrt(dv2) < 1e-9) {
+            if (sqrt(dr2) < P.d) {
+                Conj cj;
+                cj.i = cd.i; cj.j = cd.j; cj.step = cd.step; cj.flags = 2u;  // CD_FLAG_DEGENERATE
+                cj.tca = tk; cj.pca = sqrt(dr2);
+                append(out, ocap, &ctrl->n_conj, cj);
+            }
+            continue;
+        }
+        const double h = 0.5 * P.dt;
+        double tau = -(dr[0] * dv[0] + dr[1] * dv[1] + dr[2] * dv[2]) / dv2;
+        tau = fmin(fmax(tau, -h), h);
+        const double lx = fma(tau, dv[0], dr[0]), ly = fma(tau, dv[1], dr[1]), lz = fma(tau, dv[2], dr[2]);
+        const double dl = sqrt(lx * lx + ly * ly + lz * lz);
+        const double qi = O.at(kQper, cd.i), qj = O.at(kQper, cd.j);
+        const double amax = kMu / (qi * qi) + kMu / (qj * qj);
+        const double margin = 0.625 * amax * h * h + 1e-6;
+        if (dl - margin >= P.d) continue;
+        const double vi2 = vi[0] * vi[0] + vi[1] * vi[1] + vi[2] * vi[2];
+        const double vj2 = vj[0] * vj[0] + vj[1] * vj[1] + vj[2] * vj[2];
+        Work it;
+        it.i = cd.i; it.j = cd.j; it.step = cd.step; it.pad = 0;
+        it.tw = 2.0 * P.gc / sqrt(fmin(vi2, vj2));
+        append(w, wcap, n_work, it);
+    }
+}
+
+__device__ __forceinline__ double dist2_at(const Orbits& O, uint32_t i, uint32_t j, double t)
+{
+    double a[3], b[3], v[3];
+    state<false>(O, i, t, a, v);
+    state<false>(O, j, t, b, v);
+    const double dx = a[0] - b[0], dy = a[1] - b[1], dz = a[2] - b[2];
+    return fma(dx, dx, fma(dy, dy, dz * dz));
+}
+
+__global__ void __launch_bounds__(128) k_brent(Orbits O, RefineParams P, const Work* __restrict__ w,
+                                               const unsigned long long* n_work, size_t wcap,
+                                               Conj* __restrict__ out, size_t ocap, Ctrl* ctrl)
+{
+    unsigned long long nw = *n_work;
+    if (nw > wcap) nw = wcap;
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < nw; idx += stride) {
+        const Work it = w[idx];
+        const double tk = fma((double)it.step, P.dt, P.t0);
+        double a = fmax(-it.tw, P.t0 - tk);
+        double b = fmin(it.tw, P.t1 - tk);
+        if (!(b > a)) continue;
+        const double lo = a, hi = b;
+        // Brent's localmin (golden section + successive parabolic interpolation)
+        const double cgold = 0.3819660112501051;   // (3 - sqrt 5)/2
+        const double eps = 1.4901161193847656e-08; // sqrt(2^-52)
+        const double tabs = 1e-9;                  // absolute tolerance in tau [s]
+        double x = a + cgold * (b - a), wv = x, vv = x;
+        double fx = dist2_at(O, it.i, it.j, tk + x), fw = fx, fv = fx;
+        double d = 0.0, e = 0.0;
+        for (int iter = 0; iter < 100; ++iter) {
+            const double m = 0.5 * (a + b);
+            const double tol = eps * fabs(x) + tabs;
+            const double t2 = 2.0 * tol;
+            if (fabs(x - m) <= t2 - 0.5 * (b - a)) break;
+            double pp = 0.0, qq = 0.0, rr = 0.0;
+            if (fabs(e) > tol) {
+                rr = (x - wv) * (fx - fv);
+                qq = (x - vv) * (fx - fw);
+                pp = (x - vv) * qq - (x - wv) * rr;
+                qq = 2.0 * (qq - rr);
+                if (qq > 0.0) pp = -pp;
+                else qq = -qq;
+                rr = e;
+                e = d;
+            }
+            if (fabs(pp) < fabs(0.5 * qq * rr) && pp > qq * (a - x) && pp < qq * (b - x)) {
+                d = pp / qq;
+                const double u = x + d;
+                if ((u - a) < t2 || (b - u) < t2) d = (x < m) ? tol : -tol;
+            } else {
+                e = (x < m) ? b - x : a - x;
+                d = cgold * e;
+            }
+            const double u = x + (fabs(d) >= tol ? d : (d > 0.0 ? tol : -tol));
+            const double fu = dist2_at(O, it.i, it.j, tk + u);
+            if (fu <= fx) {
+                if (u < x) b = x;
+                else a = x;
+                vv = wv; fv = fw; wv = x; fw = fx; x = u; fx = fu;
+            } else {
+                if (u < x) a = u;
+                else b = u;
+                if (fu <= fw || wv == x) {
+                    vv = wv; fv = fw; wv = u; fw = fu;
+                } else if (fu <= fv || vv == x || vv == wv) {
+                    vv = u; fv = fu;
+                }
+            }
+        }
+        // interval-edge rule
+        const double tol = eps * fabs(x) + tabs;
+        if (x - lo <= 3.0 * tol || hi - x <= 3.0 * tol) continue;
+        const double tca = tk + x;
+        if (tca < P.t0 || tca > P.t1) continue;
+        const double kstar = floor((tca - P.t0) / P.dt + 0.5);
+        if (kstar != (double)it.step) continue;
+        const double pca = sqrt(fx);
+        if (!(pca < P.d)) continue;
+        Conj cj;
+        cj.i = it.i; cj.j = it.j; cj.step = it.step; cj.flags = 0u;
+        cj.tca = tca; cj.pca = pca;
+        append(out, ocap, &ctrl->n_conj, cj);
+    }
+}
+
+cudaError_t launch_prefilter(const Orbits& O, const RefineParams& p, const Cand* q, size_t qcap,
+                             Work* w, size_t wcap, unsigned long long* n_work, Conj* out, size_t ocap,
+                             Ctrl* ctrl, cudaStream_t st, LaunchCount& lc)
+{
+    k_prefilter<<<148 * 8, 256, 0, st>>>(O, p, q, qcap, w, wcap, n_work, out, ocap, ctrl);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_brent(const Orbits& O, const RefineParams& p, const Work* w,
+                         const unsigned long long* n_work, size_t wcap, Conj* out, size_t ocap,
+                         Ctrl* ctrl, cudaStream_t st, LaunchCount& lc)
+{
+    k_brent<<<148 * 8, 128, 0, st>>>(O, p, w, n_work, wcap, out, ocap, ctrl);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+}  // namespace cdh

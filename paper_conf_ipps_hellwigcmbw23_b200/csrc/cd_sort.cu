@@ -1,0 +1,135 @@
+// cd_sort.cu -- a10 finalize: map internal object order to the caller's ids and sort the
+// records by (i, j, step) on the device (CUB radix sort, stable, two passes), plus the
+// eccentricity-class sort used by the precompute.
+#include <cub/cub.cuh>
+
+#include "cd_internal.h"
+
+using namespace cdk;
+
+namespace cdh {
+
+#define CD_TRY(x)                                  \
+    do {                                           \
+        cudaError_t _e = (x);                      \
+        if (_e != cudaSuccess) return _e;          \
+    } while (0)
+
+template <typename T>
+static cudaError_t dalloc(T** p, size_t count, cudaStream_t st)
+{
+    return cudaMallocAsync((void**)p, sizeof(T) * (count ? count : 1), st);
+}
+
+cudaError_t sort_pairs_u32(const uint32_t* kin, uint32_t* kout, const uint32_t* vin, uint32_t* vout,
+                           size_t count, int end_bit, cudaStream_t st, LaunchCount& lc)
+{
+    size_t tmp_bytes = 0;
+    CD_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, kin, kout, vin, vout, (int64_t)count,
+                                           0, end_bit, st));
+    void* tmp = nullptr;
+    CD_TRY(cudaMallocAsync(&tmp, tmp_bytes ? tmp_bytes : 1, st));
+    CD_TRY(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, kin, kout, vin, vout, (int64_t)count, 0,
+                                           end_bit, st));
+    lc.bump(4);   // CUB onesweep: histogram + exclusive scan + one pass per 8-bit digit (upper bound)
+    return cudaFreeAsync(tmp, st);
+}
+
+template <typename Rec>
+__global__ void k_map_keys(const Rec* __restrict__ in, size_t n, const uint32_t* __restrict__ perm,
+                           uint32_t* __restrict__ step_key, uint32_t* __restrict__ idx)
+{
+    const size_t q = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
+    if (q >= n) return;
+    step_key[q] = in[q].step;
+    idx[q] = (uint32_t)q;
+}
+
+template <typename Rec>
+__global__ void k_pair_keys(const Rec* __restrict__ in, const uint32_t* __restrict__ idx, size_t n,
+                            const uint32_t* __restrict__ perm, unsigned long long* __restrict__ key)
+{
+    const size_t q = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
+    if (q >= n) return;
+    const Rec r = in[idx[q]];
+    uint32_t a = perm[r.i], b = perm[r.j];
+    if (a > b) { uint32_t t = a; a = b; b = t; }
+    key[q] = ((unsigned long long)a << 32) | b;
+}
+
+template <typename Rec>
+__global__ void k_gather(const Rec* __restrict__ in, const uint32_t* __restrict__ idx, size_t n,
+                         const uint32_t* __restrict__ perm, Rec* __restrict__ out)
+{
+    const size_t q = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
+    if (q >= n) return;
+    Rec r = in[idx[q]];
+    uint32_t a = perm[r.i], b = perm[r.j];
+    if (a > b) { uint32_t t = a; a = b; b = t; }
+    r.i = a;
+    r.j = b;
+    out[q] = r;
+}
+
+template <typename Rec>
+static cudaError_t finalize_impl(const Rec* in, size_t n, const uint32_t* perm, Rec* out,
+                                 cudaStream_t st, LaunchCount& lc)
+{
+    if (n == 0) return cudaSuccess;
+    if (n >= (size_t(1) << 32)) return cudaErrorInvalidValue;
+    uint32_t *k1 = nullptr, *k1o = nullptr, *i1 = nullptr, *i1o = nullptr, *i2o = nullptr;
+    unsigned long long *k2 = nullptr, *k2o = nullptr;
+    CD_TRY(dalloc(&k1, n, st));
+    CD_TRY(dalloc(&k1o, n, st));
+    CD_TRY(dalloc(&i1, n, st));
+    CD_TRY(dalloc(&i1o, n, st));
+    CD_TRY(dalloc(&i2o, n, st));
+    CD_TRY(dalloc(&k2, n, st));
+    CD_TRY(dalloc(&k2o, n, st));
+    const unsigned blocks = (unsigned)((n + 255) / 256);
+    // pass 1: by step
+    k_map_keys<Rec><<<blocks, 256, 0, st>>>(in, n, perm, k1, i1);
+    lc.bump();
+    CD_TRY(cudaGetLastError());
+    size_t tb = 0;
+    CD_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, k1, k1o, i1, i1o, (int64_t)n, 0, 32, st));
+    size_t tb2 = 0;
+    CD_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb2, k2, k2o, i1o, i2o, (int64_t)n, 0, 64, st));
+    if (tb2 > tb) tb = tb2;
+    void* tmp = nullptr;
+    CD_TRY(cudaMallocAsync(&tmp, tb ? tb : 1, st));
+    CD_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, k1, k1o, i1, i1o, (int64_t)n, 0, 32, st));
+    lc.bump(6);
+    // pass 2 (stable): by (i, j) in caller ids
+    k_pair_keys<Rec><<<blocks, 256, 0, st>>>(in, i1o, n, perm, k2);
+    lc.bump();
+    CD_TRY(cudaGetLastError());
+    CD_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, k2, k2o, i1o, i2o, (int64_t)n, 0, 64, st));
+    lc.bump(10);
+    k_gather<Rec><<<blocks, 256, 0, st>>>(in, i2o, n, perm, out);
+    lc.bump();
+    CD_TRY(cudaGetLastError());
+    cudaFreeAsync(tmp, st);
+    cudaFreeAsync(k1, st);
+    cudaFreeAsync(k1o, st);
+    cudaFreeAsync(i1, st);
+    cudaFreeAsync(i1o, st);
+    cudaFreeAsync(i2o, st);
+    cudaFreeAsync(k2, st);
+    cudaFreeAsync(k2o, st);
+    return cudaGetLastError();
+}
+
+cudaError_t finalize_conj(const Conj* in, size_t count, const uint32_t* perm, Conj* out,
+                          cudaStream_t st, LaunchCount& lc)
+{
+    return finalize_impl<Conj>(in, count, perm, out, st, lc);
+}
+
+cudaError_t finalize_cand(const Cand* in, size_t count, const uint32_t* perm, Cand* out,
+                          cudaStream_t st, LaunchCount& lc)
+{
+    return finalize_impl<Cand>(in, count, perm, out, st, lc);
+}
+
+}  // namespace cdh

@@ -1,0 +1,88 @@
+"""Parity comparison between the CUDA path and the oracle (SURVEY.md 8(c) parity rules).
+
+* candidates: identical (i, j, k) sets, excluding only triples whose distance at t_k lies within
+  1 mm of g_c (either side);
+* conjunctions: identical (i, j, step) sets excluding rows with |PCA - d| < 1 mm, TCA within
+  1e-3 s of an owner-cell boundary t_k +- dt/2 or of t0 / t1, or the oracle's MULTI flag; matched
+  rows need |dTCA| <= 1e-3 s and |dPCA| <= 1 m.
+"""
+from __future__ import annotations
+
+import math
+from collections import defaultdict
+
+import numpy as np
+
+import oracle
+
+MM = 1e-6          # 1 mm in km
+TCA_TOL = 1e-3     # s
+PCA_TOL = 1e-3     # km (1 m)
+
+
+def _keys(a):
+    return set(zip(a["i"].tolist(), a["j"].tolist(), a["step"].tolist()))
+
+
+def compare_candidates(pop, gpu, orc, t0, dt, gc):
+    """Returns the number of excluded (boundary) triples; asserts everything else matches."""
+    g, o = _keys(gpu), _keys(orc)
+    diff = sorted(g ^ o)
+    for (i, j, k) in diff:
+        tk = t0 + k * dt
+        D, _ = oracle.pair_distance(pop, i, j, [tk])
+        assert abs(D[0] - gc) < MM, (f"candidate ({i},{j},{k}) only in "
+                                     f"{'gpu' if (i, j, k) in g else 'oracle'}: D = {D[0]!r}, "
+                                     f"g_c = {gc}")
+    assert len(gpu) == len(g), "duplicate candidates in the GPU output"
+    return len(diff)
+
+
+def _excluded_row(r, t0, t1, dt, d):
+    if abs(r["pca"] - d) < MM:
+        return True
+    tk = t0 + int(r["step"]) * dt
+    for b in (tk - 0.5 * dt, tk + 0.5 * dt, t0, t1):
+        if abs(r["tca"] - b) < TCA_TOL:
+            return True
+    return False
+
+
+def compare_conjunctions(pop, gpu, orc, t0, t1, dt, d, gc):
+    """Returns dict(matched, excluded); asserts the parity rules."""
+    G = defaultdict(list)
+    O = defaultdict(list)
+    for r in gpu:
+        G[(int(r["i"]), int(r["j"]), int(r["step"]))].append(r)
+    for r in orc:
+        O[(int(r["i"]), int(r["j"]), int(r["step"]))].append(r)
+    # MULTI status of every key (oracle predicate)
+    keys = sorted(set(G) | set(O))
+    cand = np.array(keys, dtype=np.uint32).reshape(-1, 3)
+    ca = np.zeros(len(keys), dtype=oracle.CAND_DTYPE)
+    if len(keys):
+        ca["i"], ca["j"], ca["step"] = cand[:, 0], cand[:, 1], cand[:, 2]
+    flags = dict(zip(keys, oracle.candidate_flags(pop, t0, dt, gc, ca).tolist())) if len(keys) else {}
+    matched = excluded = 0
+    for k in keys:
+        g, o = G.get(k, []), O.get(k, [])
+        if flags[k] & oracle.MULTI or any(_excluded_row(r, t0, t1, dt, d) for r in g + o):
+            excluded += 1
+            continue
+        assert len(g) == 1 and len(o) == 1, (k, g, o)
+        g, o = g[0], o[0]
+        assert abs(g["tca"] - o["tca"]) <= TCA_TOL, (k, g, o)
+        assert abs(g["pca"] - o["pca"]) <= PCA_TOL, (k, g, o)
+        assert bool(g["flags"] & 2) == bool(o["flags"] & 2), (k, g, o)
+        matched += 1
+    assert len(gpu) == 0 or np.all(gpu["i"] < gpu["j"])
+    return {"matched": matched, "excluded": excluded}
+
+
+def is_sorted(a):
+    if len(a) < 2:
+        return True
+    k = np.stack([a["i"].astype(np.int64), a["j"].astype(np.int64), a["step"].astype(np.int64)], 1)
+    d = np.diff(k, axis=0)
+    first = np.where(d[:, 0] != 0, d[:, 0], np.where(d[:, 1] != 0, d[:, 1], d[:, 2]))
+    return bool(np.all(first >= 0))

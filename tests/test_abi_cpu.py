@@ -1,0 +1,85 @@
+"""CPU-side checks of the C-ABI library (no compute calls): it loads, exports every symbol
+include/cdscreen.h declares, its structs have the declared layout, and without a GPU every
+compute entry point fails loudly (no CPU fallback)."""
+import ctypes as C
+import re
+import subprocess
+from pathlib import Path
+
+import numpy as np
+import pytest
+
+ROOT = Path(__file__).resolve().parent.parent
+HEADER = ROOT / "include" / "cdscreen.h"
+
+
+@pytest.fixture(scope="module")
+def cds():
+    from paper_conf_ipps_hellwigcmbw23_b200 import _build
+    _build.build()
+    import paper_conf_ipps_hellwigcmbw23_b200 as m
+    m.lib()
+    return m
+
+
+def declared_functions():
+    txt = HEADER.read_text()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"^\s*(?:[A-Za-z_][\w\s\*]*?)\b(cd_\w+)\s*\(", txt, flags=re.M)))
+
+
+def test_exports_every_declared_symbol(cds):
+    names = declared_functions()
+    assert "cd_screen" in names and "cd_propagate" in names and len(names) >= 11
+    out = subprocess.run(["nm", "-D", "--defined-only", str(cds.LIB_PATH)], capture_output=True,
+                         text=True, check=True).stdout
+    exported = set(re.findall(r"\b(cd_\w+)\b", out))
+    missing = [n for n in names if n not in exported]
+    assert not missing, missing
+    L = cds.lib()
+    for n in names:
+        assert hasattr(L, n)
+    assert set(names) == set(cds.ABI_SYMBOLS)
+
+
+def test_version_status_options(cds):
+    assert cds.cd_abi_version() == 1
+    assert cds.status_str(cds.CD_EINVAL) == "CD_EINVAL"
+    assert cds.status_str(cds.CD_ENODEV) == "CD_ENODEV"
+    o = cds.cd_options()
+    cds.cd_options_init(o)
+    assert o.v_margin == 7.8 and o.n_ranks == 1 and o.cell_factor == 1.0 and o.device == -1
+
+
+def test_struct_layouts(cds):
+    assert C.sizeof(cds.cd_conjunction) == 32 and cds.CONJ_DTYPE.itemsize == 32
+    assert C.sizeof(cds.cd_candidate) == 12 and cds.CAND_DTYPE.itemsize == 12
+    assert C.sizeof(cds.cd_elements) == 48
+
+
+def _has_gpu():
+    try:
+        import torch
+        return torch.cuda.is_available()
+    except Exception:
+        return False
+
+
+@pytest.mark.skipif(_has_gpu(), reason="checks the no-GPU behaviour")
+def test_no_cpu_fallback(cds):
+    pop = {k: np.ones(4) * v for k, v in zip(cds.FIELDS, (7000.0, 0.001, 1, 1, 1, 1))}
+    with pytest.raises(cds.CdError) as ei:
+        cds.screen(pop, 0.0, 10.0, 1.0, 2.0)
+    assert ei.value.status == cds.CD_ENODEV
+    with pytest.raises(cds.CdError) as ei:
+        cds.propagate(pop, [0.0])
+    assert ei.value.status == cds.CD_ENODEV
+
+
+def test_product_never_imports_oracle():
+    pkg = ROOT / "paper_conf_ipps_hellwigcmbw23_b200"
+    for p in list(pkg.rglob("*.py")) + list(pkg.rglob("*.cu")) + list(pkg.rglob("*.cuh")) + \
+            list(pkg.rglob("*.h")) + [HEADER]:
+        txt = p.read_text()
+        assert "import oracle" not in txt and "from oracle" not in txt, p
+        assert "cd_oracle" not in txt and "liborc" not in txt, p
