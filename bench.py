@@ -1,0 +1,381 @@
+#!/usr/bin/env python
+"""Benchmark of the B200-native screening path (BASELINE.json metric: object-steps/s and wall
+time for the 1M-object x 24 h screen at 1/2/4/8 B200).
+
+Workload: BASELINE.json config 4 (1,000,000 objects, d = 2 km, 24 h window, grid variant at
+dt = 1 s -> 86,401 sampling steps; the hybrid variant at dt = 9 s is reported alongside).
+A bench "step" is one pass of the whole hot path (precompute, propagate + insert, neighbour scan,
+refinement, finalize) over one time slice of that window: the timed steps x N ranks slices
+partition the 24 h window exactly (owner rule, no overlap), so the timed region screens the
+whole day once at every N (strong scaling) and ``value`` = 1e6 x 86,401 / max-over-ranks time.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+from pathlib import Path
+
+import numpy as np
+
+ROOT = Path(__file__).resolve().parent
+sys.path.insert(0, str(ROOT))
+
+ALG_BYTES = {"scan": 248.0, "insert": 48.0, "propagate": 0.0, "clear": 16.0}   # SURVEY.md 8(d), per object-step
+FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12                        # 37.2 TFLOP/s
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def load_peaks():
+    p = ROOT / "MEASURED_PEAKS.json"
+    if p.exists():
+        d = json.loads(p.read_text())
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region (B200_PROFILING.md)."""
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,"
+                 "clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+                 "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_power_cap", "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm = []
+        mx = None
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            try:
+                sm.append(float(r[0]))
+                mx = float(r[1])
+                for nm, v in zip(names, r[3:7]):
+                    if v.lower().startswith("active"):
+                        reasons.add(nm)
+            except Exception:
+                continue
+        load = [x for x in sm if x > 500] or sm
+        return {"sm_mhz": float(np.median(load)) if load else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def population(args):
+    from tools import popgen
+    pop, cfg, _ = popgen.make_config(args.config, n=args.n)
+    return pop, cfg
+
+
+def cpu_oracle_sample(pop, cfg, dt, d, k0, nsteps):
+    """The oracle as it stands on the host cores: candidates (CPU grid) + conjunctions for
+    steps [k0, k0 + nsteps) of the window; returns (seconds, threads)."""
+    import oracle
+    gc = oracle.cell_size(d, dt)
+    t = time.perf_counter()
+    K = oracle.candidates_grid(pop, cfg.t0, cfg.t1, dt, gc, k_begin=k0, k_end=k0 + nsteps)
+    oracle.conjunctions(pop, cfg.t0, cfg.t1, dt, d, gc, K)
+    return time.perf_counter() - t, oracle.num_threads()
+
+
+def run_reference(args):
+    """--impl reference: the oracle (plain C, OpenMP) timed as it stands on the host cores, on a
+    bounded sample of the same workload per step.  Rank 0 only."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    pop, cfg = population(args)
+    n = len(pop["a"])
+    dt = cfg.dt_grid if args.variant == "grid" else cfg.dt_hybrid
+    threads = oracle.num_threads()
+    per = max(1, min(args.ref_steps or threads, 64))
+    K = oracle.num_steps(cfg.t0, cfg.t1, dt)
+    total = 0.0
+    for s in range(args.warmup + args.steps):
+        k0 = ((s * 997) * per) % max(1, K - per)
+        sec, _ = cpu_oracle_sample(pop, cfg, dt, cfg.d, k0, per)
+        if s >= args.warmup:
+            total += sec
+    units = n * per * args.steps
+    value = units / total
+    line = {"impl": "reference", "metric": "object-steps/s (1M objects x 24 h screen)",
+            "value": value, "unit": "object-steps/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": workload_config(args, cfg, n, dt, K),
+            "cpu_baseline": {"value": value, "unit": "object-steps/s", "cores": threads,
+                             "kind": "oracle",
+                             "sample": f"{per} consecutive {dt:g}-s steps of the 24 h window per "
+                                       f"bench step (CPU grid + conjunctions), {n} objects"},
+            "e2e": {"value": value, "unit": "object-steps/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def workload_config(args, cfg, n, dt, K):
+    return {"workload": f"BASELINE config {args.config}: {n} objects, d = {cfg.d:g} km, "
+                        f"{(cfg.t1 - cfg.t0) / 3600:g} h window, {args.variant} variant, "
+                        f"dt = {dt:g} s ({K} steps)",
+            "n_objects": n, "threshold_km": cfg.d, "dt_s": dt, "window_s": cfg.t1 - cfg.t0,
+            "steps_in_window": K, "variant": args.variant,
+            "population": "seeded synthetic (tools/popgen.py), paper-shaped LEO-heavy mixture "
+                          "+ Starlink-like shells",
+            "l2": "flushed between timed steps (256 MB write); working set > L2"}
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_hellwigcmbw23_b200 as cds
+    from paper_conf_ipps_hellwigcmbw23_b200 import dist as cdist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    pop, cfg = population(args)
+    n = len(pop["a"])
+    dt = cfg.dt_grid if args.variant == "grid" else cfg.dt_hybrid
+    mode = cds.CD_GRID if args.variant == "grid" else cds.CD_HYBRID
+    K = int(np.floor((cfg.t1 - cfg.t0) / dt)) + 1
+    S = args.steps * world                                   # slices of the window, timed
+    dpop = {k: torch.from_numpy(v).to(dev) for k, v in pop.items()}   # inputs resident in HBM
+    flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)   # 256 MB > L2
+    stream = torch.cuda.current_stream(dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def one_step(s, profile, host_inputs=False):
+        q = (s * world + rank) % S
+        E = cds._Elements(pop if host_inputs else dpop)
+        st = cds.cd_stats()
+        opt = cds.make_options(rank=q, n_ranks=S, device=dev.index, stream=stream.cuda_stream,
+                               inputs_on_device=not host_inputs,
+                               outputs_on_device=not host_inputs, profile_phases=profile)
+        import ctypes as C
+        opt.stats = C.pointer(st)
+        out = cds.cd_conjunctions()
+        cds._check(cds.cd_screen_ex(E.s, E.n, cfg.t0, cfg.t1, dt, cfg.d, mode, opt, out))
+        try:
+            if host_inputs:
+                nrec = int(out.count)
+                merged = nrec
+            else:
+                recs = cdist.device_records_to_tensor(out, dev)
+                if world > 1:
+                    recs = cdist.merge_conjunctions(recs, stream=stream.cuda_stream)
+                merged = recs.shape[0]
+                nrec = int(out.count)
+        finally:
+            cds.cd_conjunctions_free(out)
+        return st.as_dict(), nrec, merged
+
+    # warm-up (untimed)
+    for w in range(args.warmup):
+        one_step(w % args.steps, profile=False)
+    torch.cuda.synchronize()
+
+    # timed region: device time with CUDA events on the library's stream, max over ranks
+    launches0 = cds.cd_kernel_launches()
+    times, stats = [], []
+    nconj = 0
+    with ClockSampler(dev.index) as clk:
+        for s in range(args.steps):
+            flush.zero_()                      # L2 flush between timed steps (outside the timing)
+            torch.cuda.synchronize()
+            barrier()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            st, nrec, merged = one_step(s, profile=args.profile)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            barrier()
+            times.append(e0.elapsed_time(e1))
+            stats.append(st)
+            nconj += nrec
+    launches = cds.cd_kernel_launches() - launches0
+    tot_ms = float(np.sum(times))
+    if world > 1:
+        t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        tot_ms = float(t.item())
+        c = torch.tensor([nconj], dtype=torch.int64, device=dev)
+        dist.all_reduce(c)
+        nconj = int(c.item())
+    units = float(n) * sum(st["steps"] for st in stats) * 1.0
+    if world > 1:
+        u = torch.tensor([units], dtype=torch.float64, device=dev)
+        dist.all_reduce(u)
+        units = float(u.item())
+    value = units / (tot_ms / 1e3)
+
+    # end to end through the public API with HOST buffers (pinned inputs, results to host)
+    e2e_ms = []
+    pin = {k: torch.from_numpy(v).pin_memory() for k, v in pop.items()}
+    pin_np = {k: v.numpy() for k, v in pin.items()}
+    d2h = 0
+    for s in range(args.e2e_steps if args.e2e_steps is not None else args.steps):
+        flush.zero_()
+        torch.cuda.synchronize()
+        barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        q = (s * world + rank) % S
+        recs = cds.screen(pin_np, cfg.t0, cfg.t1, dt, cfg.d, mode=args.variant, rank=q, n_ranks=S,
+                          device=dev.index, stream=stream.cuda_stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms.append(e0.elapsed_time(e1))
+        d2h += recs.nbytes
+    ne2e = len(e2e_ms)
+    e2e_tot = float(np.sum(e2e_ms))
+    if world > 1:
+        t = torch.tensor([e2e_tot], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_tot = float(t.item())
+    e2e_units = float(n) * (K / S) * ne2e * world
+    e2e = {"value": e2e_units / (e2e_tot / 1e3), "unit": "object-steps/s",
+           "h2d_bytes_per_step": 48 * n, "d2h_bytes_per_step": int(d2h / max(1, ne2e)),
+           "steps": ne2e}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return 0
+
+    # roofline of the dominant kernel (live CUDA-event phase times inside the timed region)
+    hbm_peak, peak_kind = load_peaks()
+    roof = None
+    if args.profile:
+        ph = {"scan": ("ms_scan", "launches_scan"),
+              "propagate": ("ms_propagate", "launches_propagate"),
+              "insert": ("ms_insert", "launches_insert"),
+              "clear": ("ms_clear", "launches_clear")}
+        ms = {k: sum(s[a] for s in stats) for k, (a, _) in ph.items()}
+        ms["refine"] = sum(s["ms_refine"] for s in stats)
+        dom = max(ms, key=ms.get)
+        if dom in ALG_BYTES:
+            nl = sum(s[ph[dom][1]] for s in stats)
+            objsteps = sum(s["object_steps"] for s in stats)
+            per_launch_bytes = ALG_BYTES[dom] * objsteps / max(1, nl)
+            avg_s = ms[dom] / 1e3 / max(1, nl)
+            achieved = per_launch_bytes / avg_s / 1e9
+            roof = {"kernel": {"scan": "k_scan", "propagate": "k_propagate", "insert": "k_insert",
+                               "clear": "k_fill_u64"}[dom],
+                    "bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+                    "frac": achieved / hbm_peak, "traffic": traffic_from_profiles(dom),
+                    "peak_source": peak_kind,
+                    "alg_bytes_per_object_step": ALG_BYTES[dom],
+                    "avg_launch_ms": 1e3 * avg_s, "launches": nl,
+                    "phase_share": {k: v / max(1e-9, sum(ms.values())) for k, v in ms.items()}}
+        else:
+            roof = {"kernel": "k_brent", "bound": "alu", "phase_share": ms}
+
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        k0 = 43200
+        per = args.cpu_steps
+        sec, threads = cpu_oracle_sample(pop, cfg, dt, cfg.d, k0, per)
+        cpu = {"value": n * per / sec, "unit": "object-steps/s", "cores": threads, "kind": "oracle",
+               "sample": f"steps [{k0}, {k0 + per}) of the same 24 h window ({per} x {n} "
+                         f"object-steps: CPU grid candidates + conjunctions), {sec:.1f} s"}
+
+    line = {"metric": "object-steps/s (1M objects x 24 h screen)", "value": value,
+            "unit": "object-steps/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": tot_ms / args.steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": dict(workload_config(args, cfg, n, dt, K),
+                           slices=S, wall_s_window=tot_ms / 1e3 * (S / (args.steps * world)),
+                           conjunctions=nconj, parallelism=f"time-slice x{world}"),
+            "clocks": clk.summary(), "e2e": e2e, "gpu_launches": launches,
+            "roofline": roof, "cpu_baseline": cpu}
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def traffic_from_profiles(phase):
+    """dram bytes per launch of the dominant kernel from the committed ncu summary, or None."""
+    p = ROOT / "profiles" / "ncu_summary.json"
+    if not p.exists():
+        return None
+    try:
+        d = json.loads(p.read_text())
+        return d.get(phase, {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=24)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--variant", default="grid", choices=["grid", "hybrid"])
+    ap.add_argument("--config", type=int, default=4)
+    ap.add_argument("--n", type=int, default=None, help="override object count (testing)")
+    ap.add_argument("--no-profile", dest="profile", action="store_false")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-steps", type=int, default=16)
+    ap.add_argument("--ref-steps", type=int, default=None)
+    ap.add_argument("--e2e-steps", type=int, default=None)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        log("note: --warmup < 3 violates the timing rules; using 3")
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

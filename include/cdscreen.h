@@ -104,8 +104,10 @@ typedef struct {
     uint64_t kernel_launches;  /* CUDA kernels launched by this call                          */
     uint64_t retries;          /* capacity-overflow retries                                   */
     double ms_total;           /* device time of the call (CUDA events on the call's stream)  */
-    double ms_propagate_insert, ms_scan, ms_refine, ms_finalize; /* per-phase device time (only
-                                  when cd_options.profile_phases != 0; adds syncs)            */
+    /* per-phase device time and launch counts, filled only when cd_options.profile_phases != 0
+       (CUDA events recorded on the call's stream around every launch; no extra syncs)         */
+    double ms_clear, ms_propagate, ms_insert, ms_scan, ms_refine, ms_finalize, ms_precompute;
+    uint64_t launches_clear, launches_propagate, launches_insert, launches_scan, launches_refine;
 } cd_stats;
 
 typedef struct {
@@ -122,7 +124,9 @@ typedef struct {
     double cell_factor;       /* grid cell edge = cell_factor * g_c (>= 1); default 1 (paper)  */
     size_t batch_object_steps;/* object-steps per in-flight step batch; 0 = auto              */
     size_t round_steps;       /* steps per refinement round; 0 = auto                         */
-    int profile_phases;       /* fill cd_stats per-phase times (serialises phases)            */
+    int profile_phases;       /* fill cd_stats per-phase times (CUDA events per launch)        */
+    int l2_persist;           /* pin the per-step grid in a persisting-L2 window (default 1;
+                                 raises cudaLimitPersistingL2CacheSize for the device)         */
     cd_stats* stats;          /* optional output                                              */
 } cd_options;
 
@@ -153,6 +157,11 @@ cd_status cd_candidates(const cd_elements* el, size_t n, double t0, double t1, d
  * are caller-owned host buffers of nt*n*3 doubles, layout [time][object][x,y,z]. */
 cd_status cd_propagate(const cd_elements* el, size_t n, const double* t, size_t nt, double* xyz,
                        double* vxyz, const cd_options* opt /* nullable */);
+
+/* Sort n conjunction records that live in device memory by (i, j, step), in place, on `stream`
+ * (cudaStream_t; NULL = the legacy default stream).  Used to merge per-rank time slices after
+ * an all-gather.  Requires i < j in every record. */
+cd_status cd_conjunctions_sort_device(cd_conjunction* data, size_t n, void* stream);
 
 void cd_conjunctions_free(cd_conjunctions* c);
 void cd_candidates_free(cd_candidate* c);

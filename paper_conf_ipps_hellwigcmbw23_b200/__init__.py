@@ -30,7 +30,7 @@ CAND_DTYPE = np.dtype([("i", "<u4"), ("j", "<u4"), ("step", "<u4")])
 
 # C ABI symbols declared in include/cdscreen.h
 ABI_SYMBOLS = ("cd_options_init", "cd_screen", "cd_screen_ex", "cd_candidates", "cd_propagate",
-               "cd_conjunctions_free", "cd_candidates_free", "cd_status_str", "cd_last_error",
+               "cd_conjunctions_sort_device", "cd_conjunctions_free", "cd_candidates_free", "cd_status_str", "cd_last_error",
                "cd_abi_version", "cd_kernel_launches")
 
 
@@ -63,8 +63,12 @@ class cd_stats(C.Structure):
                 ("hybrid_ap_rejected", C.c_uint64), ("hybrid_coplanar", C.c_uint64),
                 ("hybrid_path_rejected", C.c_uint64), ("hybrid_time_rejected", C.c_uint64),
                 ("kernel_launches", C.c_uint64), ("retries", C.c_uint64),
-                ("ms_total", C.c_double), ("ms_propagate_insert", C.c_double),
-                ("ms_scan", C.c_double), ("ms_refine", C.c_double), ("ms_finalize", C.c_double)]
+                ("ms_total", C.c_double), ("ms_clear", C.c_double),
+                ("ms_propagate", C.c_double), ("ms_insert", C.c_double),
+                ("ms_scan", C.c_double), ("ms_refine", C.c_double), ("ms_finalize", C.c_double),
+                ("ms_precompute", C.c_double), ("launches_clear", C.c_uint64),
+                ("launches_propagate", C.c_uint64), ("launches_insert", C.c_uint64),
+                ("launches_scan", C.c_uint64), ("launches_refine", C.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -76,7 +80,8 @@ class cd_options(C.Structure):
                 ("inputs_on_device", C.c_int), ("outputs_on_device", C.c_int),
                 ("kepler_points", C.c_int), ("cell_factor", C.c_double),
                 ("batch_object_steps", C.c_size_t), ("round_steps", C.c_size_t),
-                ("profile_phases", C.c_int), ("stats", C.POINTER(cd_stats))]
+                ("profile_phases", C.c_int), ("l2_persist", C.c_int),
+                ("stats", C.POINTER(cd_stats))]
 
 
 _lib = None
@@ -106,6 +111,8 @@ def lib():
         L.cd_propagate.restype = C.c_int
         L.cd_propagate.argtypes = [P(cd_elements), C.c_size_t, C.c_void_p, C.c_size_t, C.c_void_p,
                                    C.c_void_p, P(cd_options)]
+        L.cd_conjunctions_sort_device.restype = C.c_int
+        L.cd_conjunctions_sort_device.argtypes = [C.c_void_p, C.c_size_t, C.c_void_p]
         L.cd_conjunctions_free.restype = None
         L.cd_conjunctions_free.argtypes = [P(cd_conjunctions)]
         L.cd_candidates_free.restype = None
@@ -157,6 +164,10 @@ def cd_propagate(el, n, t, nt, xyz, vxyz, opt):
                               C.byref(opt) if opt is not None else None)
 
 
+def cd_conjunctions_sort_device(ptr, n, stream):
+    return lib().cd_conjunctions_sort_device(ptr, n, stream)
+
+
 def cd_conjunctions_free(c):
     lib().cd_conjunctions_free(C.byref(c))
 
@@ -194,7 +205,8 @@ class _Elements:
 
 def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None, stream=None,
                  cell_factor=None, batch_object_steps=None, round_steps=None,
-                 outputs_on_device=False, inputs_on_device=False):
+                 outputs_on_device=False, inputs_on_device=False, profile_phases=False,
+                 l2_persist=None):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -215,6 +227,9 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
         o.round_steps = int(round_steps)
     o.outputs_on_device = int(bool(outputs_on_device))
     o.inputs_on_device = int(bool(inputs_on_device))
+    o.profile_phases = int(bool(profile_phases))
+    if l2_persist is not None:
+        o.l2_persist = int(bool(l2_persist))
     return o
 
 

@@ -108,6 +108,78 @@ struct Owner {
     void* p;
 };
 
+// Optional per-phase device timing (cd_options.profile_phases): CUDA events recorded on the
+// call's stream around each launch; elapsed times are harvested after the round's sync.
+enum Phase { kPhClear = 0, kPhPropagate, kPhInsert, kPhScan, kPhRefine, kPhFinalize, kPhPrecompute, kNPhase };
+
+struct PhaseTimer {
+    bool on = false;
+    cudaStream_t st = nullptr;
+    std::vector<cudaEvent_t> pool;
+    size_t used = 0;
+    struct Mark { int ph; size_t a, b; };
+    std::vector<Mark> marks;
+    double ms[kNPhase] = {};
+    uint64_t launches[kNPhase] = {};
+    int cur = -1;
+    size_t cur_a = 0;
+    ~PhaseTimer()
+    {
+        for (auto e : pool) cudaEventDestroy(e);
+    }
+    cudaEvent_t ev()
+    {
+        if (used == pool.size()) {
+            cudaEvent_t e;
+            cudaEventCreate(&e);
+            pool.push_back(e);
+        }
+        return pool[used++];
+    }
+    void start(int ph)
+    {
+        if (!on) return;
+        cur = ph;
+        cur_a = used;
+        cudaEventRecord(ev(), st);
+    }
+    void stop()
+    {
+        if (!on || cur < 0) return;
+        const size_t b = used;
+        cudaEventRecord(ev(), st);
+        marks.push_back({cur, cur_a, b});
+        cur = -1;
+    }
+    // call after the stream has been synchronised
+    void harvest()
+    {
+        if (!on) return;
+        for (const Mark& m : marks) {
+            float x = 0.f;
+            if (cudaEventElapsedTime(&x, pool[m.a], pool[m.b]) == cudaSuccess) ms[m.ph] += x;
+            launches[m.ph] += 1;
+        }
+        marks.clear();
+        used = 0;
+    }
+    void to_stats(cd_stats& s) const
+    {
+        s.ms_clear = ms[kPhClear];
+        s.ms_propagate = ms[kPhPropagate];
+        s.ms_insert = ms[kPhInsert];
+        s.ms_scan = ms[kPhScan];
+        s.ms_refine = ms[kPhRefine];
+        s.ms_finalize = ms[kPhFinalize];
+        s.ms_precompute = ms[kPhPrecompute];
+        s.launches_clear = launches[kPhClear];
+        s.launches_propagate = launches[kPhPropagate];
+        s.launches_insert = launches[kPhInsert];
+        s.launches_scan = launches[kPhScan];
+        s.launches_refine = launches[kPhRefine];
+    }
+};
+
 // One library call: device, stream, events, launch count.
 struct Call {
     int prev_dev = -1, dev = -1;
@@ -115,6 +187,7 @@ struct Call {
     bool own_stream = false;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     LaunchCount lc;
+    PhaseTimer pt;
     ~Call()
     {
         if (ev0) cudaEventDestroy(ev0);
@@ -149,6 +222,8 @@ struct Call {
         CU(cudaEventCreate(&ev0));
         CU(cudaEventCreate(&ev1));
         CU(cudaEventRecord(ev0, st));
+        pt.on = o.profile_phases != 0;
+        pt.st = st;
         return CD_OK;
     }
 };
@@ -241,6 +316,7 @@ cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_opti
             CU(cudaMemcpyAsync(up.p + c * n, src[c], sizeof(double) * n, cudaMemcpyHostToDevice, st));
         E = Elements{up.p, up.p + n, up.p + 2 * n, up.p + 3 * n, up.p + 4 * n, up.p + 5 * n};
     }
+    C.pt.start(kPhPrecompute);
     DBuf<uint32_t> key(st), idx(st), keyo(st);
     CU(key.alloc(n));
     CU(idx.alloc(n));
@@ -251,6 +327,7 @@ cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_opti
     CU(S.rec.alloc((size_t)kNCol * n));
     CU(S.cls.alloc(n));
     CU(launch_build_records(E, S.perm.p, (int64_t)n, S.rec.p, S.cls.p, st, C.lc));
+    C.pt.stop();
     return CD_OK;
 }
 
@@ -290,21 +367,62 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     g.oz = o.grid_origin[2];
     g.inv_cell = 1.0 / L;
     g.gc2 = gc * gc;
+    g.reach = gc * (1.0 + 1e-9) + 1e-9;
+    g.halfshell = L < 2.0 * gc ? 1 : 0;
     RefineParams P{t0, t1, dt, d, gc};
 
     R.conj.st = R.cand.st = st;
     if (ke <= kb || n < 2) return CD_OK;
 
-    const uint64_t M = next_pow2((uint64_t)std::max<int64_t>(2 * n, 64));   // 2n slots
+    const uint64_t M = next_pow2((uint64_t)std::max<int64_t>(2 * n, 64));   // >= 2n slots (power of 2)
     const uint64_t mask = M - 1;
     const size_t target = o.batch_object_steps ? o.batch_object_steps : (size_t(1) << 20);
     int64_t Bmax = std::max<int64_t>(1, (int64_t)(target / (size_t)n));
     Bmax = std::min<int64_t>(Bmax, std::min<int64_t>(ke - kb, 65535));
 
-    DBuf<Slot> tabs(st);
-    DBuf<Entry> ents(st);
-    CU(tabs.alloc((size_t)Bmax * M));
-    CU(ents.alloc((size_t)Bmax * n));
+    // per-step grid arena: two ping-pong table sets [slots | occupancy bitmap] x Bmax, then the
+    // entries; batch b builds set b & 1 while its scan zeroes set (b + 1) & 1
+    const uint64_t nbits = std::max<uint64_t>(next_pow2((uint64_t)n * 32), 1024);   // >= 32 bits/object
+    const uint32_t bwords = (uint32_t)(nbits / 32);
+    const size_t slot_bytes = sizeof(Slot) * (size_t)Bmax * M;
+    const size_t bit_bytes = ((sizeof(uint32_t) * (size_t)Bmax * bwords + 255) / 256) * 256;
+    const size_t set_bytes = slot_bytes + bit_bytes;
+    const size_t ent_bytes = sizeof(Entry) * (size_t)Bmax * n;
+    DBuf<unsigned char> arena(st);
+    CU(arena.alloc(2 * set_bytes + ent_bytes));
+    CU(cudaMemsetAsync(arena.p, 0, 2 * set_bytes, st));
+    GridTab tabs[2];
+    for (int h = 0; h < 2; ++h) {
+        unsigned char* base = arena.p + h * set_bytes;
+        tabs[h] = GridTab{reinterpret_cast<Slot*>(base), reinterpret_cast<uint32_t*>(base + slot_bytes),
+                          (uint32_t)(nbits - 1), bwords};
+    }
+    Entry* ents = reinterpret_cast<Entry*>(arena.p + 2 * set_bytes);
+    uint64_t batch_no = 0;
+    // persisting-L2 window over the table set being built/scanned (slots + bitmap): these take the
+    // random atomics and probes, while records, entries and the zeroing stream past them
+    L2Win wins[2];
+    if (o.l2_persist) {
+        int maxwin = 0, maxpersist = 0;
+        cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, C.dev);
+        cudaDeviceGetAttribute(&maxpersist, cudaDevAttrMaxPersistingL2CacheSize, C.dev);
+        if (maxwin > 0 && maxpersist > 0) {
+            size_t cur = 0;
+            cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+            const size_t setaside = std::min<size_t>((size_t)maxpersist, set_bytes);
+            if (cur < setaside) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside);
+            cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+            for (int h = 0; h < 2; ++h) {
+                wins[h].on = cur > 0;
+                wins[h].w.base_ptr = arena.p + h * set_bytes;
+                wins[h].w.num_bytes = std::min<size_t>(set_bytes, (size_t)maxwin);
+                wins[h].w.hitRatio = (float)std::min(1.0, (double)cur / (double)wins[h].w.num_bytes);
+                wins[h].w.hitProp = cudaAccessPropertyPersisting;
+                wins[h].w.missProp = cudaAccessPropertyStreaming;
+            }
+        }
+        cudaGetLastError();   // persistence is best effort
+    }
     size_t qcap = std::max<size_t>(size_t(1) << 22, 4 * (size_t)n);
     DBuf<Cand> q(st);
     CU(q.alloc(qcap));
@@ -339,12 +457,20 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         CU(cudaMemsetAsync(nwork.p, 0, sizeof(unsigned long long), st));
         for (int64_t kk = k; kk < k + Rk; kk += Bmax) {
             const int B = (int)std::min<int64_t>(Bmax, k + Rk - kk);
-            CU(launch_fill_u64(reinterpret_cast<unsigned long long*>(tabs.p), (size_t)B * M * 2,
-                               ~0ull, st, C.lc));
-            CU(launch_prop_insert(O, g, tabs.p, ents.p, mask, kk, B, t0, dt, ctrl.p, st, C.lc));
-            CU(launch_scan(g, tabs.p, ents.p, n, mask, kk, B, q.p, qcap, ctrl.p, st, C.lc));
+            const GridTab& cur = tabs[batch_no & 1];
+            const GridTab& nxt = tabs[(batch_no + 1) & 1];
+            C.pt.start(kPhPropagate);
+            const L2Win* win = &wins[batch_no & 1];
+            CU(launch_prop_insert(O, g, cur, ents, mask, kk, B, t0, dt, ctrl.p, win, st, C.lc));
+            C.pt.stop();
+            C.pt.start(kPhScan);
+            CU(launch_scan(g, cur, nxt, (int)Bmax, ents, n, mask, kk, kKeyTag, B, q.p, qcap, ctrl.p,
+                           win, st, C.lc));
+            C.pt.stop();
+            ++batch_no;
         }
         if (want == Want::Conj) {
+            C.pt.start(kPhRefine);
             if (mode == CD_HYBRID) {
                 CU(launch_hybrid_filter(O, P, q.p, qcap, w.p, wcap, nwork.p, R.conj.p, ocap, ctrl.p,
                                         st, C.lc));
@@ -354,10 +480,14 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                                     C.lc));
                 CU(launch_brent(O, P, w.p, nwork.p, wcap, R.conj.p, ocap, ctrl.p, st, C.lc));
             }
+            C.pt.stop();
         }
         CU(cudaMemcpyAsync(hctrl, ctrl.p, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
         CU(cudaMemcpyAsync(hnwork, nwork.p, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
         CU(cudaStreamSynchronize(st));
+        C.pt.harvest();
+        if (hctrl->err_internal)
+            return fail(CD_EINTERNAL, "internal: a grid cell list did not terminate");
         if (hctrl->err_range)
             return fail(CD_ERANGE, "a position fell outside the cell-key range (+-%lld cells of %g km)",
                         (long long)kCellMax, L);
@@ -462,8 +592,10 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
         else if (!el) return fail(CD_EINVAL, "elements must be non-NULL");
         TRY(run(C, S, t0, t1, dt, d, mode, o, K, Want::Conj, R, stats));
         if (R.n_conj) {
+            C.pt.start(kPhFinalize);
             CU(sorted.alloc(R.n_conj));
             CU(finalize_conj(R.conj.p, R.n_conj, S.perm.p, sorted.p, C.st, C.lc));
+            C.pt.stop();
         }
     }
     Owner* own = new Owner{o.outputs_on_device != 0, nullptr};
@@ -487,6 +619,8 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
     stats.ms_total = ms;
     stats.conjunctions = R.n_conj;
     stats.kernel_launches = C.lc.n;
+    C.pt.harvest();
+    C.pt.to_stats(stats);
     if (o.stats) *o.stats = stats;
     out->data = static_cast<cd_conjunction*>(own->p);
     out->count = R.n_conj;
@@ -507,6 +641,7 @@ void cd_options_init(cd_options* o)
     o->rank = 0;
     o->n_ranks = 1;
     o->cell_factor = 1.0;
+    o->l2_persist = 1;
 }
 
 cd_status cd_screen(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,
@@ -604,6 +739,23 @@ cd_status cd_propagate(const cd_elements* el, size_t n, const double* t, size_t 
             s.kernel_launches = C.lc.n;
             *o.stats = s;
         }
+        return CD_OK;
+    } catch (...) {
+        return fail(CD_EINTERNAL, "unexpected C++ exception");
+    }
+}
+
+cd_status cd_conjunctions_sort_device(cd_conjunction* data, size_t n, void* stream)
+{
+    try {
+        if (n == 0) return CD_OK;
+        if (!data) return fail(CD_EINVAL, "data must be non-NULL");
+        cudaStream_t st = (cudaStream_t)stream;
+        LaunchCount lc;
+        DBuf<Conj> tmp(st);
+        CU(tmp.alloc(n));
+        CU(finalize_conj(reinterpret_cast<const Conj*>(data), n, nullptr, tmp.p, st, lc));
+        CU(cudaMemcpyAsync(data, tmp.p, sizeof(Conj) * n, cudaMemcpyDeviceToDevice, st));
         return CD_OK;
     } catch (...) {
         return fail(CD_EINTERNAL, "unexpected C++ exception");

@@ -44,7 +44,9 @@ struct Orbits {
     const double* rec;   // kNCol x n
     const uint8_t* cls;  // eccentricity class per object
     int64_t n;
-    __device__ __forceinline__ double at(int c, int64_t r) const { return __ldg(rec + c * n + r); }
+    // records are streamed once per step: evict-first so they do not push the per-step grid
+    // (slots, bitmap, entries) out of L2
+    __device__ __forceinline__ double at(int c, int64_t r) const { return __ldcs(rec + c * n + r); }
 };
 
 // ---------------------------------------------------------------------------------------
@@ -155,7 +157,17 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
     const double c = M + dc;
     double sc, cc;
     sincos(c, &sc, &cc);
-    const double ecr = O.at(kEcr, r), esr = O.at(kEsr, r);
+    double ecr, esr;
+    if (N == 4) {
+        // class 0 (e <= 0.01, rho <= 0.005): the six per-object constants are evaluated here by
+        // short Taylor series (truncation < 1e-22) instead of being streamed from the records
+        const double x2 = rho * rho;
+        ecr = e * fma(fma(fma(-1.0 / 720.0, x2, 1.0 / 24.0), x2, -0.5), x2, 1.0);
+        esr = e * rho * fma(fma(fma(-1.0 / 5040.0, x2, 1.0 / 120.0), x2, -1.0 / 6.0), x2, 1.0);
+    } else {
+        ecr = O.at(kEcr, r);
+        esr = O.at(kEsr, r);
+    }
     // real nodes th = 0 (z = c + rho) and th = pi (z = c - rho)
     const double f0 = (dc + rho) - (sc * ecr + cc * esr);
     const double fp = (dc - rho) - (sc * ecr - cc * esr);
@@ -172,10 +184,20 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
             constexpr int cl = N == 4 ? 0 : N == 6 ? 1 : N == 8 ? 2 : N == 12 ? 3 : 4;
             const double ct = kNodes[cl][j - 1][0], st = kNodes[cl][j - 1][1];
             const double c2t = kNodes[cl][j - 1][2], s2t = kNodes[cl][j - 1][3];
-            const double ec = O.at(kTab + 4 * (j - 1) + 0, r);
-            const double es = O.at(kTab + 4 * (j - 1) + 1, r);
-            const double ch = O.at(kTab + 4 * (j - 1) + 2, r);
-            const double sh = O.at(kTab + 4 * (j - 1) + 3, r);
+            double ec, es, ch, sh;
+            if (N == 4) {   // th = pi/3: rho cos th = rho/2, rho sin th = rho sqrt(3)/2
+                const double a = 0.5 * rho, a2 = a * a;
+                const double b = 0.86602540378443864676 * rho, b2 = b * b;
+                ec = e * fma(fma(fma(-1.0 / 720.0, a2, 1.0 / 24.0), a2, -0.5), a2, 1.0);
+                es = e * a * fma(fma(fma(-1.0 / 5040.0, a2, 1.0 / 120.0), a2, -1.0 / 6.0), a2, 1.0);
+                ch = fma(fma(fma(1.0 / 720.0, b2, 1.0 / 24.0), b2, 0.5), b2, 1.0);
+                sh = b * fma(fma(fma(1.0 / 5040.0, b2, 1.0 / 120.0), b2, 1.0 / 6.0), b2, 1.0);
+            } else {
+                ec = O.at(kTab + 4 * (j - 1) + 0, r);
+                es = O.at(kTab + 4 * (j - 1) + 1, r);
+                ch = O.at(kTab + 4 * (j - 1) + 2, r);
+                sh = O.at(kTab + 4 * (j - 1) + 3, r);
+            }
             // point j (cos th = +ct) and its mirror N-1-j (cos th = -ct, same sin th)
             const double esin_a = sc * ec + cc * es, ecos_a = cc * ec - sc * es;
             const double esin_b = sc * ec - cc * es, ecos_b = cc * ec + sc * es;
@@ -198,24 +220,39 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
     cE = fma(cc, cd, -sc * sd);
 }
 
+// Classes 1-4 (e > 0.01, a small minority of the LEO-heavy populations) live out of line so
+// the register allocation of the hot class-0 path (N = 4) stays small.
+static __device__ __noinline__ void kepler_solve_slow(double M, double e, int cls, Orbits O, int64_t r,
+                                               double* E, double* sE, double* cE)
+{
+    switch (cls) {
+    case 1: contour_core<6>(M, e, O, r, *E, *sE, *cE); break;
+    case 2: contour_core<8>(M, e, O, r, *E, *sE, *cE); break;
+    case 3: contour_core<12>(M, e, O, r, *E, *sE, *cE); break;
+    default: {
+        contour_core<16>(M, e, O, r, *E, *sE, *cE);
+        // e > 0.6: Newton polish of the contour estimate (DESIGN.md R15)
+        for (int it = 0; it < 8; ++it) {
+            const double dE = (*E - e * *sE - M) / (1.0 - e * *cE);
+            *E -= dE;
+            sincos(*E, sE, cE);
+            if (fabs(dE) <= 1e-15 * fmax(1.0, fabs(*E))) break;
+        }
+    }
+    }
+}
+
 __device__ __forceinline__ void kepler_solve(double M, double e, int cls, const Orbits& O,
                                              int64_t r, double& E, double& sE, double& cE)
 {
-    switch (cls) {
-    case 0: contour_core<4>(M, e, O, r, E, sE, cE); break;
-    case 1: contour_core<6>(M, e, O, r, E, sE, cE); break;
-    case 2: contour_core<8>(M, e, O, r, E, sE, cE); break;
-    case 3: contour_core<12>(M, e, O, r, E, sE, cE); break;
-    default: {
-        contour_core<16>(M, e, O, r, E, sE, cE);
-        // e > 0.6: Newton polish of the contour estimate (DESIGN.md R15)
-        for (int it = 0; it < 8; ++it) {
-            const double dE = (E - e * sE - M) / (1.0 - e * cE);
-            E -= dE;
-            sincos(E, &sE, &cE);
-            if (fabs(dE) <= 1e-15 * fmax(1.0, fabs(E))) break;
-        }
-    }
+    if (cls == 0) {
+        contour_core<4>(M, e, O, r, E, sE, cE);
+    } else {
+        double e_, s_, c_;
+        kepler_solve_slow(M, e, cls, O, r, &e_, &s_, &c_);
+        E = e_;
+        sE = s_;
+        cE = c_;
     }
 }
 
@@ -243,14 +280,18 @@ __device__ __forceinline__ void state(const Orbits& O, int64_t r, double t, doub
 // ---------------------------------------------------------------------------------------
 // grid cells and keys ("calculates the grid cell based on the Cartesian coordinates")
 // ---------------------------------------------------------------------------------------
-constexpr int64_t kKeyBias = int64_t(1) << 20;
+// Cell keys pack 19 bits per axis (cells in [-(2^18 - 2), 2^18 - 2], i.e. +-262,142 cells of
+// edge L >= g_c: +-46,000 km at g_c = 0.18 km); the top 7 bits of a stored key word hold a
+// non-zero tag so a stored key is never the all-zero empty value.
+constexpr int64_t kKeyBias = int64_t(1) << 18;
 constexpr int64_t kCellMax = kKeyBias - 2;   // valid cells in [-kCellMax, kCellMax]
-constexpr uint64_t kEmpty = ~uint64_t(0);    // the maximum 64-bit value marks empty
+constexpr int kTagShift = 57;
+constexpr uint32_t kKeyTag = 1;
 constexpr uint32_t kNil = 0xffffffffu;
 
 __device__ __forceinline__ uint64_t pack_key(int64_t cx, int64_t cy, int64_t cz)
 {
-    return uint64_t(cx + kKeyBias) | (uint64_t(cy + kKeyBias) << 21) | (uint64_t(cz + kKeyBias) << 42);
+    return uint64_t(cx + kKeyBias) | (uint64_t(cy + kKeyBias) << 19) | (uint64_t(cz + kKeyBias) << 38);
 }
 
 // MurmurHash3 64-bit finaliser (footnote 3: smhasher)
@@ -266,8 +307,11 @@ __device__ __forceinline__ uint64_t fmix64(uint64_t k)
 
 struct GridGeom {
     double ox, oy, oz;   // origin
-    double inv_cell;     // 1 / cell edge
+    double inv_cell;     // 1 / cell edge L (L >= g_c)
     double gc2;          // g_c^2 (candidate gate)
+    double reach;        // g_c (1 + 1e-9) + 1e-9: ball radius used to pick the probed cells
+    int halfshell;       // 1: own cell + 13 half-shell neighbours (L < 2 g_c); 0: the cells
+                         // overlapping the ball |x - p| < g_c (L >= 2 g_c)
 };
 
 __device__ __forceinline__ bool cell_of(const GridGeom& g, const double p[3], int64_t c[3])
@@ -286,12 +330,96 @@ struct __align__(32) Entry {
     uint32_t pad;
 };
 
-// Hash-map slot: 64-bit cell key + head of the cell's entry list.
+// Hash grid of one step.  Open addressing over M = 2^m >= 2n slots,
+// linear probing s_{i+1} = s_i + 1 mod M (Eq. 2) from the MurmurHash3 slot.  A slot is
+// 16 bytes {cell key | tag, list head}: key and head are installed together by one 128-bit CAS
+// (P:147-148's CAS, widened so that claiming a cell and pushing the first object onto its list is
+// a single atomic).  An all-zero slot is empty (P:147 reserves one value for "empty"; zero lets
+// tables be cleared with plain coalesced stores); keys carry a non-zero tag in their top bits.
 struct __align__(16) Slot {
-    unsigned long long key;
-    uint32_t head;
-    uint32_t pad;
+    unsigned long long key;    // pack_key(cell) | tag << 57
+    unsigned long long head;   // low 32 bits: entry index of the list head (Fig. 6)
 };
+
+__device__ __forceinline__ bool cas128(Slot* s, unsigned long long& e0, unsigned long long& e1,
+                                       unsigned long long d0, unsigned long long d1)
+{
+    unsigned long long o0, o1;
+    asm volatile("{ .reg .b128 d, b, c;\n\t"
+                 "mov.b128 b, {%2, %3};\n\t"
+                 "mov.b128 c, {%4, %5};\n\t"
+                 "atom.relaxed.gpu.global.cas.b128 d, [%6], b, c;\n\t"
+                 "mov.b128 {%0, %1}, d; }"
+                 : "=l"(o0), "=l"(o1)
+                 : "l"(e0), "l"(e1), "l"(d0), "l"(d1), "l"(s)
+                 : "memory");
+    const bool ok = o0 == e0 && o1 == e1;
+    e0 = o0;
+    e1 = o1;
+    return ok;
+}
+
+// Non-blocking insert of object r into the cell `key`.  Tables are zeroed before
+// each use, so the first attempt on a slot is a blind CAS against the empty value {0, 0}: claiming
+// an empty cell costs one atomic; a slot already holding the key pushes r onto its list (CAS of
+// the head); a slot of another cell moves on along the probe sequence (Eq. 2).  Returns the
+// previous list head (r's `next`), kNil if r is the first object of its cell.
+__device__ __forceinline__ uint32_t grid_insert(Slot* slots, uint64_t mask, unsigned long long key,
+                                                uint32_t tag, uint32_t r)
+{
+    const unsigned long long tk = key | ((unsigned long long)tag << kTagShift);
+    uint64_t h = fmix64(key) & mask;
+    unsigned long long e0 = 0ull, e1 = 0ull;
+    while (true) {
+        if (cas128(slots + h, e0, e1, tk, (unsigned long long)r))
+            return e0 == 0ull ? kNil : (uint32_t)e1;
+        // failed: (e0, e1) = current contents
+        if (e0 != tk) {   // another cell (the slot cannot return to empty): next slot
+            h = (h + 1) & mask;
+            e0 = 0ull;
+            e1 = 0ull;
+        }
+        // same cell: retry the push with the observed head
+    }
+}
+
+// Per-step occupancy bitmap over hashed cell keys: 32 bits per object, so a probe of an empty
+// cell (the common case) is one 4-byte load from a 4 MB (at 1M objects) L2-resident array;
+// false positives (~3 %) only cost a table probe.  MurmurHash3 fmix32 of the folded key.
+__device__ __forceinline__ uint32_t fmix32(uint32_t h)
+{
+    h ^= h >> 16;
+    h *= 0x85ebca6bu;
+    h ^= h >> 13;
+    h *= 0xc2b2ae35u;
+    h ^= h >> 16;
+    return h;
+}
+__device__ __forceinline__ uint32_t bit_of(unsigned long long key)
+{
+    return fmix32((uint32_t)key + 0x9e3779b9u * (uint32_t)(key >> 32));
+}
+
+struct GridTab {
+    Slot* slots;      // M slots per step
+    uint32_t* bits;   // bwords words per step
+    uint32_t bmask;   // bit index mask (2^b - 1)
+    uint32_t bwords;
+};
+
+// Lookup after the build (read-only): list head of cell `key`, kNil if the cell is empty.
+__device__ __forceinline__ uint32_t grid_find(const Slot* __restrict__ slots, uint64_t mask,
+                                              unsigned long long key, uint32_t tag)
+{
+    const unsigned long long tk = key | ((unsigned long long)tag << kTagShift);
+    uint64_t h = fmix64(key) & mask;
+    while (true) {
+        const ulonglong2 w = __ldg(reinterpret_cast<const ulonglong2*>(slots + h));
+        if (w.x == tk) return (uint32_t)w.y;
+        if ((uint32_t)(w.x >> kTagShift) != tag) return kNil;
+        h = (h + 1) & mask;
+    }
+}
 
 struct Cand {   // candidate ("the satellites' ids and the sampling step")
     uint32_t i, j, step;
@@ -308,7 +436,7 @@ struct Ctrl {   // device-side counters and flags of one call
     unsigned long long n_refined;
     unsigned long long n_ap, n_coplanar, n_path, n_time;
     int err_range;
-    int pad;
+    int err_internal;
 };
 
 }  // namespace cdk

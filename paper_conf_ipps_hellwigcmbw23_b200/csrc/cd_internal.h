@@ -28,6 +28,13 @@ struct Work {
     double tw;   // Brent half-window t_w = 2 g_c / min(|v_i|, |v_j|)
 };
 
+// Optional persisting-L2 window applied to a launch (the per-step grid arena: slots, bitmap,
+// entries), so the random-access structures stay resident while the orbit records stream.
+struct L2Win {
+    bool on = false;
+    cudaAccessPolicyWindow w{};
+};
+
 struct RefineParams {
     double t0, t1, dt, d, gc;
 };
@@ -44,12 +51,16 @@ cudaError_t launch_propagate_out(const cdk::Orbits& O, const uint32_t* perm, con
 // ---- grid build + scan (a2-a6) ---------------------------------------------------------
 cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long long v,
                             cudaStream_t st, LaunchCount& lc);
-cudaError_t launch_prop_insert(const cdk::Orbits& O, const cdk::GridGeom& g, cdk::Slot* tabs,
+// Fused propagate + cell key + insert; the tables of `tab` must be zero on entry.
+cudaError_t launch_prop_insert(const cdk::Orbits& O, const cdk::GridGeom& g, const cdk::GridTab& tab,
                                cdk::Entry* ents, uint64_t mask, int64_t k0, int B, double t0,
-                               double dt, cdk::Ctrl* ctrl, cudaStream_t st, LaunchCount& lc);
-cudaError_t launch_scan(const cdk::GridGeom& g, const cdk::Slot* tabs, const cdk::Entry* ents,
-                        int64_t n, uint64_t mask, int64_t k0, int B, cdk::Cand* q, size_t qcap,
-                        cdk::Ctrl* ctrl, cudaStream_t st, LaunchCount& lc);
+                               double dt, cdk::Ctrl* ctrl, const L2Win* win, cudaStream_t st,
+                               LaunchCount& lc);
+// Neighbour scan of the batch in `tab`; also zeroes the ping-pong set `clr` for the next batch.
+cudaError_t launch_scan(const cdk::GridGeom& g, const cdk::GridTab& tab, const cdk::GridTab& clr,
+                        int nclr, const cdk::Entry* ents, int64_t n, uint64_t mask, int64_t k0, uint32_t tag,
+                        int B, cdk::Cand* q, size_t qcap, cdk::Ctrl* ctrl, const L2Win* win,
+                        cudaStream_t st, LaunchCount& lc);
 
 // ---- refinement (a7) -------------------------------------------------------------------
 cudaError_t launch_prefilter(const cdk::Orbits& O, const RefineParams& p, const cdk::Cand* q,

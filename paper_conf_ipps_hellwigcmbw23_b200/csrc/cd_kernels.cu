@@ -18,6 +18,27 @@ std::atomic<uint64_t> g_launches{0};
 
 static inline unsigned blocks_for(int64_t n, int t) { return (unsigned)((n + t - 1) / t); }
 
+// Launch with an optional persisting-L2 access-policy window (per-launch attribute).
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_ex(void (*kern)(KArgs...), dim3 grid, dim3 block, cudaStream_t st,
+                             const L2Win* win, Args... args)
+{
+    if (!win || !win->on) {
+        kern<<<grid, block, 0, st>>>(args...);
+        return cudaGetLastError();
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeAccessPolicyWindow;
+    at[0].val.accessPolicyWindow = win->w;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, args...);
+}
+
 // Warp-aggregated append: one atomicAdd per group of converged lanes.  The counter keeps
 // counting past `cap` so the host can detect overflow and size the retry.
 template <typename T>
@@ -154,15 +175,14 @@ cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long l
 }
 
 // ---------------------------------------------------------------------------------------
-// a2-a4: one thread per (object, step): propagate (Contour), cell key, non-blocking insert.
-// Insertion: 64-bit CAS of the cell key into the first empty slot of its linear
-// probe sequence s_{i+1} = s_i + 1 mod M (Eq. 2); a slot already holding the same key is the
-// same cell, so the object is pushed onto that cell's singly linked list with an atomic
-// exchange of the list head (entries pre-allocated, one per object).
+// a2-a4: one thread per (object, step) ("one thread per tuple"): Contour Kepler solve and
+// Cartesian position, cell key, non-blocking insert into the step's hash grid (P:135-150,
+// Eq. 2) and its occupancy bitmap; the entry {x, y, z, next} (Fig. 6) is written once,
+// coalesced.
 // ---------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) k_prop_insert(Orbits O, GridGeom g, Slot* __restrict__ tabs,
-                                                     Entry* __restrict__ ents, uint64_t mask,
-                                                     int64_t k0, double t0, double dt, Ctrl* ctrl)
+__global__ void __launch_bounds__(256, 4) k_prop_insert(Orbits O, GridGeom g, GridTab tab,
+                                                        Entry* __restrict__ ents, uint64_t mask,
+                                                        int64_t k0, double t0, double dt, Ctrl* ctrl)
 {
     const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (r >= O.n) return;
@@ -171,17 +191,12 @@ __global__ void __launch_bounds__(256) k_prop_insert(Orbits O, GridGeom g, Slot*
     double p[3], v[3];
     state<false>(O, r, t, p, v);
     int64_t c[3];
-    uint32_t prev = kNil;
+    uint32_t next = kNil;
     if (cell_of(g, p, c)) {
-        Slot* tab = tabs + (size_t)s * (mask + 1);
         const unsigned long long key = pack_key(c[0], c[1], c[2]);
-        uint64_t h = fmix64(key) & mask;
-        while (true) {
-            const unsigned long long old = atomicCAS(&tab[h].key, (unsigned long long)kEmpty, key);
-            if (old == kEmpty || old == key) break;
-            h = (h + 1) & mask;
-        }
-        prev = atomicExch(&tab[h].head, (uint32_t)r);
+        const uint32_t hb = bit_of(key) & tab.bmask;
+        atomicOr(tab.bits + (size_t)s * tab.bwords + (hb >> 5), 1u << (hb & 31));
+        next = grid_insert(tab.slots + (size_t)s * (mask + 1), mask, key, kKeyTag, (uint32_t)r);
     } else {
         ctrl->err_range = 1;
     }
@@ -189,28 +204,22 @@ __global__ void __launch_bounds__(256) k_prop_insert(Orbits O, GridGeom g, Slot*
     en.x = p[0];
     en.y = p[1];
     en.z = p[2];
-    en.next = prev;
+    en.next = next;
     en.pad = 0;
     ents[(size_t)s * O.n + r] = en;
 }
 
-cudaError_t launch_prop_insert(const Orbits& O, const GridGeom& g, Slot* tabs, Entry* ents,
-                               uint64_t mask, int64_t k0, int B, double t0, double dt, Ctrl* ctrl,
-                               cudaStream_t st, LaunchCount& lc)
-{
-    dim3 grid(blocks_for(O.n, 256), (unsigned)B);
-    k_prop_insert<<<grid, 256, 0, st>>>(O, g, tabs, ents, mask, k0, t0, dt, ctrl);
-    lc.bump();
-    return cudaGetLastError();
-}
-
 // ---------------------------------------------------------------------------------------
-// a5-a6: neighbour scan.  One thread per (object, step).  The object's own cell and the 13
-// cells of the positive half-shell are probed, which visits every unordered pair of cells in
-// a 3x3x3 neighbourhood exactly once ("every other satellite in that cell or the
-// 3^3-1 = 26 neighbor cells"; "prevent considering possible conjunctions twice").
-// A pair is a candidate iff |r_i - r_j| < g_c (reading R6); candidates are appended to the
-// queue with one atomic per group of converged lanes.
+// a5-a6: neighbour scan, one thread per (object, step).
+//  (1) own cell: walk the object's own list successors -- every same-cell pair is seen exactly
+//      once, by the later-inserted object (no probe needed);
+//  (2) other cells: half-shell mode (L < 2 g_c, the paper's cell g_c) probes the 13
+//      positive half-shell neighbours -- each unordered pair of cells of a 3x3x3 block once;
+//      ball mode (L >= 2 g_c) probes the 0-7 other cells overlapping |x - p| < g_c -- a pair is
+//      seen from both objects and reported by the smaller index.  The first slot of every probe
+//      is loaded before any is resolved, so a thread's probes overlap in flight.
+// A pair is a candidate iff |r_i - r_j| < g_c (reading R6); candidates are appended with one
+// atomic per group of converged lanes (P:95 saves ids + sampling step).
 // ---------------------------------------------------------------------------------------
 __constant__ int8_t kHalfShell[14][3] = {
     {0, 0, 0},
@@ -218,62 +227,133 @@ __constant__ int8_t kHalfShell[14][3] = {
     {0, 1, -1}, {0, 1, 0}, {0, 1, 1},
     {0, 0, 1}};
 
-__device__ __forceinline__ uint32_t probe(const Slot* __restrict__ tab, uint64_t mask,
-                                         unsigned long long key)
+__device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_t j, const double p[3],
+                                          const Entry& ej, uint32_t step, Cand* __restrict__ q,
+                                          size_t qcap, Ctrl* ctrl)
 {
-    uint64_t h = fmix64(key) & mask;
-    while (true) {
-        const ulonglong2 sl = __ldg(reinterpret_cast<const ulonglong2*>(tab + h));
-        if (sl.x == key) return (uint32_t)sl.y;
-        if (sl.x == kEmpty) return kNil;
-        h = (h + 1) & mask;
+    const double dx = p[0] - ej.x, dy = p[1] - ej.y, dz = p[2] - ej.z;
+    if (fma(dx, dx, fma(dy, dy, dz * dz)) < g.gc2) {
+        Cand cd;
+        cd.i = r < j ? r : j;
+        cd.j = r < j ? j : r;
+        cd.step = step;
+        append(q, qcap, &ctrl->n_cand, cd);
     }
 }
 
-__global__ void __launch_bounds__(256) k_scan(GridGeom g, const Slot* __restrict__ tabs,
-                                              const Entry* __restrict__ ents, int64_t n, uint64_t mask,
-                                              int64_t k0, Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
+__device__ __forceinline__ void walk(const GridGeom& g, const Entry* __restrict__ E, uint32_t j,
+                                     uint32_t r, const double p[3], bool only_greater, uint32_t step,
+                                     Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
+{
+    while (j != kNil) {
+        const Entry ej = E[j];
+        if (!only_greater || j > r) test_pair(g, r, j, p, ej, step, q, qcap, ctrl);
+        j = ej.next;
+    }
+}
+
+// Probe NP cells: issue every bitmap load first (independent 4-byte loads), then probe the
+// table only for set bits and walk the hits.
+template <int NP, typename KeyFn>
+__device__ __forceinline__ void probe_group(const GridGeom& g, const Slot* __restrict__ slots,
+                                            const uint32_t* __restrict__ bits, uint32_t bmask,
+                                            uint64_t mask, uint32_t tag, uint32_t valid, KeyFn keyf,
+                                            const Entry* __restrict__ E, uint32_t r, const double p[3],
+                                            bool only_greater, uint32_t step, Cand* __restrict__ q,
+                                            size_t qcap, Ctrl* ctrl)
+{
+    uint32_t hit = 0;
+#pragma unroll
+    for (int i = 0; i < NP; ++i) {
+        if ((valid >> i) & 1u) {
+            const uint32_t hb = bit_of(keyf(i)) & bmask;
+            hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << i;
+        }
+    }
+    while (hit) {
+        const int i = __ffs(hit) - 1;
+        hit &= hit - 1;
+        walk(g, E, grid_find(slots, mask, keyf(i), tag), r, p, only_greater, step, q, qcap, ctrl);
+    }
+}
+
+__global__ void __launch_bounds__(256, 1) k_scan(GridGeom g, GridTab tab, GridTab clr, int nclr,
+                                                 const Entry* __restrict__ ents, int64_t n,
+                                                 uint64_t mask, int64_t k0, uint32_t tag,
+                                                 Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
 {
     const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (r >= n) return;
     const int s = blockIdx.y;
-    const Slot* tab = tabs + (size_t)s * (mask + 1);
+    // side job: zero the other (ping-pong) table set for the next batch -- tables s, s + B, ...
+    // below nclr (the allocated batch depth), so a deeper next batch also finds zeroed tables
+    {
+        const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+        const int64_t nth = (int64_t)gridDim.x * blockDim.x;
+        for (int ss = s; ss < nclr; ss += (int)gridDim.y) {
+            // streaming stores (evict-first): the zeroed set is not touched until the next batch
+            ulonglong2* cs = reinterpret_cast<ulonglong2*>(clr.slots + (size_t)ss * (mask + 1));
+            for (int64_t i = tid; i <= (int64_t)mask; i += nth) __stcs(cs + i, make_ulonglong2(0ull, 0ull));
+            uint4* cb = reinterpret_cast<uint4*>(clr.bits + (size_t)ss * clr.bwords);
+            for (int64_t i = tid; i < (int64_t)(clr.bwords / 4); i += nth) __stcs(cb + i, make_uint4(0u, 0u, 0u, 0u));
+        }
+    }
+    if (r >= n) return;
+    const Slot* slots = tab.slots + (size_t)s * (mask + 1);
+    const uint32_t* bits = tab.bits + (size_t)s * tab.bwords;
     const Entry* E = ents + (size_t)s * n;
+    const uint32_t step = (uint32_t)(k0 + s);
     const Entry me = E[r];
     const double p[3] = {me.x, me.y, me.z};
     int64_t c[3];
     if (!cell_of(g, p, c)) return;
-    const uint32_t step = (uint32_t)(k0 + s);
-#pragma unroll 1
-    for (int o = 0; o < 14; ++o) {
-        const unsigned long long key =
-            pack_key(c[0] + kHalfShell[o][0], c[1] + kHalfShell[o][1], c[2] + kHalfShell[o][2]);
-        uint32_t j = probe(tab, mask, key);
-        while (j != kNil) {
-            const Entry ej = E[j];
-            if (o != 0 || j > (uint32_t)r) {
-                const double dx = p[0] - ej.x, dy = p[1] - ej.y, dz = p[2] - ej.z;
-                if (fma(dx, dx, fma(dy, dy, dz * dz)) < g.gc2) {
-                    Cand cd;
-                    cd.i = (uint32_t)r < j ? (uint32_t)r : j;
-                    cd.j = (uint32_t)r < j ? j : (uint32_t)r;
-                    cd.step = step;
-                    append(q, qcap, &ctrl->n_cand, cd);
-                }
-            }
-            j = ej.next;
-        }
+    // (1) own cell: successors in the object's own list
+    walk(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
+    // (2) other cells
+    if (g.halfshell) {
+        auto k1 = [=](int i) { return pack_key(c[0] + kHalfShell[1 + i][0], c[1] + kHalfShell[1 + i][1],
+                                               c[2] + kHalfShell[1 + i][2]); };
+        auto k2 = [=](int i) { return pack_key(c[0] + kHalfShell[8 + i][0], c[1] + kHalfShell[8 + i][1],
+                                               c[2] + kHalfShell[8 + i][2]); };
+        probe_group<7>(g, slots, bits, tab.bmask, mask, tag, 0x7Fu, k1, E, (uint32_t)r, p, false, step, q, qcap, ctrl);
+        probe_group<6>(g, slots, bits, tab.bmask, mask, tag, 0x3Fu, k2, E, (uint32_t)r, p, false, step, q, qcap, ctrl);
+    } else {
+        int64_t lo[3], hi[3];
+        const double pl[3] = {p[0] - g.reach, p[1] - g.reach, p[2] - g.reach};
+        const double ph[3] = {p[0] + g.reach, p[1] + g.reach, p[2] + g.reach};
+        if (!cell_of(g, pl, lo) || !cell_of(g, ph, hi)) return;
+        // per axis: the other overlapped cell (c - 1 or c + 1), or none
+        const int64_t d0 = lo[0] < c[0] ? -1 : (hi[0] > c[0] ? 1 : 0);
+        const int64_t d1 = lo[1] < c[1] ? -1 : (hi[1] > c[1] ? 1 : 0);
+        const int64_t d2 = lo[2] < c[2] ? -1 : (hi[2] > c[2] ? 1 : 0);
+        // cell c + (b0 d0, b1 d1, b2 d2), b = 1..7 (bit i <-> b = i + 1), exists iff every axis set
+        // in b has d != 0
+        const uint32_t valid = (((d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu)) >> 1) & 0x7Fu;
+        auto kb = [=](int i) {
+            const int b = i + 1;
+            return pack_key(c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0), c[2] + ((b & 4) ? d2 : 0));
+        };
+        probe_group<7>(g, slots, bits, tab.bmask, mask, tag, valid, kb, E, (uint32_t)r, p, true, step, q, qcap, ctrl);
     }
 }
 
-cudaError_t launch_scan(const GridGeom& g, const Slot* tabs, const Entry* ents, int64_t n,
-                        uint64_t mask, int64_t k0, int B, Cand* q, size_t qcap, Ctrl* ctrl,
-                        cudaStream_t st, LaunchCount& lc)
+cudaError_t launch_prop_insert(const Orbits& O, const GridGeom& g, const GridTab& tab, Entry* ents,
+                               uint64_t mask, int64_t k0, int B, double t0, double dt, Ctrl* ctrl,
+                               const L2Win* win, cudaStream_t st, LaunchCount& lc)
+{
+    dim3 grid(blocks_for(O.n, 256), (unsigned)B);
+    lc.bump();
+    return launch_ex(k_prop_insert, grid, dim3(256), st, win, O, g, tab, ents, mask, k0, t0, dt, ctrl);
+}
+
+cudaError_t launch_scan(const GridGeom& g, const GridTab& tab, const GridTab& clr, int nclr,
+                        const Entry* ents, int64_t n, uint64_t mask, int64_t k0, uint32_t tag, int B,
+                        Cand* q, size_t qcap, Ctrl* ctrl, const L2Win* win, cudaStream_t st,
+                        LaunchCount& lc)
 {
     dim3 grid(blocks_for(n, 256), (unsigned)B);
-    k_scan<<<grid, 256, 0, st>>>(g, tabs, ents, n, mask, k0, q, qcap, ctrl);
     lc.bump();
-    return cudaGetLastError();
+    return launch_ex(k_scan, grid, dim3(256), st, win, g, tab, clr, nclr, ents, n, mask, k0, tag, q,
+                     qcap, ctrl);
 }
 
 // ---------------------------------------------------------------------------------------

@@ -52,7 +52,7 @@ __global__ void k_pair_keys(const Rec* __restrict__ in, const uint32_t* __restri
     const size_t q = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
     if (q >= n) return;
     const Rec r = in[idx[q]];
-    uint32_t a = perm[r.i], b = perm[r.j];
+    uint32_t a = perm ? perm[r.i] : r.i, b = perm ? perm[r.j] : r.j;
     if (a > b) { uint32_t t = a; a = b; b = t; }
     key[q] = ((unsigned long long)a << 32) | b;
 }
@@ -64,7 +64,7 @@ __global__ void k_gather(const Rec* __restrict__ in, const uint32_t* __restrict_
     const size_t q = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
     if (q >= n) return;
     Rec r = in[idx[q]];
-    uint32_t a = perm[r.i], b = perm[r.j];
+    uint32_t a = perm ? perm[r.i] : r.i, b = perm ? perm[r.j] : r.j;
     if (a > b) { uint32_t t = a; a = b; b = t; }
     r.i = a;
     r.j = b;

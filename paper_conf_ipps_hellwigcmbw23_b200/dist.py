@@ -1,0 +1,76 @@
+"""Multi-GPU time slicing and the conjunction-list merge.
+
+One process per GPU.  The window's K sampling steps are split into contiguous slices; a call
+with ``rank=q, n_ranks=S`` screens steps [floor(q K / S), floor((q + 1) K / S)) and reports only
+the minima it owns (owner rule), so slices partition the result set with no halo and no
+data-path collective.  The one real exchange is the final merge: an all-gather of the per-rank
+record counts, then of the (padded) 32-byte records, over NCCL / NVLink (``torch.distributed``
+is the plumbing), followed by the library's device sort by (i, j, step).
+"""
+from __future__ import annotations
+
+import numpy as np
+
+REC_BYTES = 32
+
+
+def slice_range(K: int, q: int, S: int):
+    """Steps owned by slice q of S (same arithmetic as the C library's rank/n_ranks)."""
+    return (K * q) // S, (K * (q + 1)) // S
+
+
+def gather_records(local, group=None):
+    """All-gather variable-length record blocks.
+
+    `local` is a uint8 tensor of shape (m, 32) on this rank's device (cuda for NCCL, cpu for
+    gloo).  Returns the concatenation over ranks (rank order), shape (sum m, 32)."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    dev = local.device
+    cnt = torch.tensor([local.shape[0]], dtype=torch.int64, device=dev)
+    counts = [torch.zeros_like(cnt) for _ in range(world)]
+    dist.all_gather(counts, cnt, group=group)
+    counts = [int(c.item()) for c in counts]
+    mx = max(counts) if counts else 0
+    if mx == 0:
+        return torch.zeros((0, REC_BYTES), dtype=torch.uint8, device=dev)
+    pad = torch.zeros((mx, REC_BYTES), dtype=torch.uint8, device=dev)
+    pad[: local.shape[0]] = local
+    bufs = [torch.empty_like(pad) for _ in range(world)]
+    dist.all_gather(bufs, pad, group=group)
+    return torch.cat([b[:c] for b, c in zip(bufs, counts)], dim=0)
+
+
+def merge_conjunctions(local, group=None, stream=None):
+    """Gather every rank's records and sort them by (i, j, step) on the device with the library
+    (cd_conjunctions_sort_device).  `local`: uint8 cuda tensor (m, 32)."""
+    import torch
+
+    from . import _check, cd_conjunctions_sort_device
+    allrec = gather_records(local, group)
+    if allrec.shape[0] and allrec.is_cuda:
+        st = stream if stream is not None else torch.cuda.current_stream().cuda_stream
+        _check(cd_conjunctions_sort_device(allrec.data_ptr(), allrec.shape[0], st))
+    return allrec
+
+
+def device_records_to_tensor(out, device):
+    """Copy a library-owned device result (cd_conjunctions with outputs_on_device) into a torch
+    uint8 tensor (m, 32) on `device`."""
+    import torch
+    from cuda.bindings import runtime as rt
+    m = int(out.count)
+    t = torch.empty((m, REC_BYTES), dtype=torch.uint8, device=device)
+    if m:
+        err, = rt.cudaMemcpyAsync(t.data_ptr(), out.data, m * REC_BYTES,
+                                  rt.cudaMemcpyKind.cudaMemcpyDeviceToDevice,
+                                  torch.cuda.current_stream(device).cuda_stream)
+        assert int(err) == 0, err
+    return t
+
+
+def records_to_numpy(t):
+    from . import CONJ_DTYPE
+    a = t.cpu().numpy()
+    return np.frombuffer(a.tobytes(), dtype=CONJ_DTYPE).copy()
