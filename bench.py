@@ -27,7 +27,8 @@ import numpy as np
 ROOT = Path(__file__).resolve().parent
 sys.path.insert(0, str(ROOT))
 
-ALG_BYTES = {"scan": 248.0, "insert": 48.0, "propagate": 0.0, "clear": 16.0}   # SURVEY.md 8(d), per object-step
+PROFILE_EVERY = 16   # time every 16th k_step launch inside the timed region
+ALG_BYTES = {"scan": 296.0}   # insert 48 + detect 248 B per object-step (k_step fuses both)
 FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12                        # 37.2 TFLOP/s
 
 
@@ -69,6 +70,12 @@ class ClockSampler:
         for line in self.proc.stdout:
             self.rows.append([x.strip() for x in line.split(",")])
 
+    def mark(self):
+        self.i0 = len(self.rows)
+
+    def mark_end(self):
+        self.i1 = len(self.rows)
+
     def __exit__(self, *a):
         if self.proc:
             self.proc.terminate()
@@ -82,7 +89,7 @@ class ClockSampler:
         mx = None
         reasons = set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in self.rows:
+        for r in self.rows[getattr(self, "i0", 0):getattr(self, "i1", None)]:
             try:
                 sm.append(float(r[0]))
                 mx = float(r[1])
@@ -215,6 +222,9 @@ def run_ours(args):
             cds.cd_conjunctions_free(out)
         return st.as_dict(), nrec, merged
 
+    # the clock sampler starts before the warm-up so its NVML start-up does not land in the
+    # timed region; only samples taken during the timed steps are summarised
+    clk = ClockSampler(dev.index).__enter__()
     # warm-up (untimed)
     for w in range(args.warmup):
         one_step(w % args.steps, profile=False)
@@ -224,7 +234,8 @@ def run_ours(args):
     launches0 = cds.cd_kernel_launches()
     times, stats = [], []
     nconj = 0
-    with ClockSampler(dev.index) as clk:
+    clk.mark()
+    if True:
         for s in range(args.steps):
             flush.zero_()                      # L2 flush between timed steps (outside the timing)
             torch.cuda.synchronize()
@@ -232,13 +243,18 @@ def run_ours(args):
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            st, nrec, merged = one_step(s, profile=args.profile)
+            st, nrec, merged = one_step(s, profile=PROFILE_EVERY if args.profile else 0)
             e1.record(stream)
             torch.cuda.synchronize()
             barrier()
             times.append(e0.elapsed_time(e1))
             stats.append(st)
             nconj += nrec
+            if os.environ.get("BENCH_VERBOSE"):
+                log(f"step {s}: {times[-1]:.1f} ms, lib {st['ms_total']:.1f} ms, cand {st['candidates']}, "
+                    f"refined {st['refined']}, retries {st['retries']}, launches {st['kernel_launches']}")
+    clk.mark_end()
+    clk.__exit__(None, None, None)
     launches = cds.cd_kernel_launches() - launches0
     tot_ms = float(np.sum(times))
     if world > 1:
@@ -294,29 +310,27 @@ def run_ours(args):
     hbm_peak, peak_kind = load_peaks()
     roof = None
     if args.profile:
-        ph = {"scan": ("ms_scan", "launches_scan"),
-              "propagate": ("ms_propagate", "launches_propagate"),
-              "insert": ("ms_insert", "launches_insert"),
-              "clear": ("ms_clear", "launches_clear")}
-        ms = {k: sum(s[a] for s in stats) for k, (a, _) in ph.items()}
-        ms["refine"] = sum(s["ms_refine"] for s in stats)
-        dom = max(ms, key=ms.get)
-        if dom in ALG_BYTES:
-            nl = sum(s[ph[dom][1]] for s in stats)
-            objsteps = sum(s["object_steps"] for s in stats)
-            per_launch_bytes = ALG_BYTES[dom] * objsteps / max(1, nl)
-            avg_s = ms[dom] / 1e3 / max(1, nl)
-            achieved = per_launch_bytes / avg_s / 1e9
-            roof = {"kernel": {"scan": "k_scan", "propagate": "k_propagate", "insert": "k_insert",
-                               "clear": "k_fill_u64"}[dom],
-                    "bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
-                    "frac": achieved / hbm_peak, "traffic": traffic_from_profiles(dom),
-                    "peak_source": peak_kind,
-                    "alg_bytes_per_object_step": ALG_BYTES[dom],
-                    "avg_launch_ms": 1e3 * avg_s, "launches": nl,
-                    "phase_share": {k: v / max(1e-9, sum(ms.values())) for k, v in ms.items()}}
-        else:
-            roof = {"kernel": "k_brent", "bound": "alu", "phase_share": ms}
+        # k_step (fused build + scan) runs as the "propagate" phase (first, build-only launch of
+        # each round) and the "scan" phase (all other launches); its algorithmic bytes are
+        # SURVEY 8(d)'s 296 B per object-step (insert 48 + detect 248)
+        # sampled: every PROFILE_EVERY-th launch of a phase is timed (events on the call's stream)
+        ms_smp = sum(s_["ms_scan"] + s_["ms_propagate"] for s_ in stats)
+        nl_smp = sum(s_["launches_scan"] + s_["launches_propagate"] for s_ in stats)
+        nl = sum(s_["step_launches"] for s_ in stats)
+        avg_s = ms_smp / 1e3 / max(1, nl_smp)
+        ms_step = 1e3 * avg_s * nl                         # estimated total k_step time
+        objsteps = sum(s_["object_steps"] for s_ in stats)
+        tot = max(1e-9, tot_ms)
+        alg = ALG_BYTES["scan"] * objsteps
+        achieved = alg / max(1, nl) / avg_s / 1e9
+        roof = {"kernel": "k_step (fused propagate + insert + neighbour scan)",
+                "bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+                "frac": achieved / hbm_peak, "traffic": traffic_from_profiles("k_step"),
+                "peak_source": peak_kind, "alg_bytes_per_object_step": ALG_BYTES["scan"],
+                "alg_bytes_per_launch": alg / max(1, nl), "avg_launch_ms": 1e3 * avg_s,
+                "launches": nl,
+                "launches_timed": nl_smp,
+                "share_of_step_time": ms_step / tot}
 
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
@@ -334,6 +348,8 @@ def run_ours(args):
             "config": dict(workload_config(args, cfg, n, dt, K),
                            slices=S, wall_s_window=tot_ms / 1e3 * (S / (args.steps * world)),
                            conjunctions=nconj, parallelism=f"time-slice x{world}"),
+            "step_ms": {"min": float(np.min(times)), "median": float(np.median(times)),
+                        "max": float(np.max(times))},
             "clocks": clk.summary(), "e2e": e2e, "gpu_launches": launches,
             "roofline": roof, "cpu_baseline": cpu}
     print(json.dumps(line), flush=True)
@@ -365,7 +381,7 @@ def main():
     ap.add_argument("--n", type=int, default=None, help="override object count (testing)")
     ap.add_argument("--no-profile", dest="profile", action="store_false")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-steps", type=int, default=16)
+    ap.add_argument("--cpu-steps", type=int, default=128)
     ap.add_argument("--ref-steps", type=int, default=None)
     ap.add_argument("--e2e-steps", type=int, default=None)
     args = ap.parse_args()

@@ -104,10 +104,12 @@ typedef struct {
     uint64_t kernel_launches;  /* CUDA kernels launched by this call                          */
     uint64_t retries;          /* capacity-overflow retries                                   */
     double ms_total;           /* device time of the call (CUDA events on the call's stream)  */
-    /* per-phase device time and launch counts, filled only when cd_options.profile_phases != 0
-       (CUDA events recorded on the call's stream around every launch; no extra syncs)         */
+    /* per-phase device time and timed-launch counts, filled only when cd_options.profile_phases
+       > 0 (CUDA events on the call's stream around every profile_phases-th launch of a phase;
+       no extra syncs): average launch duration = ms_X / launches_X                            */
     double ms_clear, ms_propagate, ms_insert, ms_scan, ms_refine, ms_finalize, ms_precompute;
     uint64_t launches_clear, launches_propagate, launches_insert, launches_scan, launches_refine;
+    uint64_t step_launches;    /* all launches of the fused step kernel (timed or not)         */
 } cd_stats;
 
 typedef struct {
@@ -121,12 +123,14 @@ typedef struct {
     int inputs_on_device;     /* element pointers are device pointers                         */
     int outputs_on_device;    /* cd_conjunctions.data stays in device memory                  */
     int kepler_points;        /* 0 = choose the Contour point count per object from e         */
-    double cell_factor;       /* grid cell edge = cell_factor * g_c (>= 1); default 1 (paper)  */
+    double cell_factor;       /* grid cell edge = cell_factor * g_c (>= 1); 1 = the paper's cell
+                                 and 27-cell scan; default 0 = auto (chosen from the measured
+                                 candidate density; results do not depend on it)               */
     size_t batch_object_steps;/* object-steps per in-flight step batch; 0 = auto              */
     size_t round_steps;       /* steps per refinement round; 0 = auto                         */
-    int profile_phases;       /* fill cd_stats per-phase times (CUDA events per launch)        */
-    int l2_persist;           /* pin the per-step grid in a persisting-L2 window (default 1;
-                                 raises cudaLimitPersistingL2CacheSize for the device)         */
+    int profile_phases;       /* N > 0: time every N-th launch of each phase into cd_stats     */
+    int l2_persist;           /* pin the per-step grid tables in a persisting-L2 window (default
+                                 0; raises cudaLimitPersistingL2CacheSize for the device)      */
     cd_stats* stats;          /* optional output                                              */
 } cd_options;
 

@@ -68,7 +68,8 @@ class cd_stats(C.Structure):
                 ("ms_scan", C.c_double), ("ms_refine", C.c_double), ("ms_finalize", C.c_double),
                 ("ms_precompute", C.c_double), ("launches_clear", C.c_uint64),
                 ("launches_propagate", C.c_uint64), ("launches_insert", C.c_uint64),
-                ("launches_scan", C.c_uint64), ("launches_refine", C.c_uint64)]
+                ("launches_scan", C.c_uint64), ("launches_refine", C.c_uint64),
+                ("step_launches", C.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -227,7 +228,7 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
         o.round_steps = int(round_steps)
     o.outputs_on_device = int(bool(outputs_on_device))
     o.inputs_on_device = int(bool(inputs_on_device))
-    o.profile_phases = int(bool(profile_phases))
+    o.profile_phases = int(profile_phases)
     if l2_persist is not None:
         o.l2_persist = int(bool(l2_persist))
     return o

@@ -123,6 +123,8 @@ struct PhaseTimer {
     uint64_t launches[kNPhase] = {};
     int cur = -1;
     size_t cur_a = 0;
+    uint64_t every = 1;               // time every `every`-th launch of a phase (sampling)
+    uint64_t calls[kNPhase] = {};     // all launches per phase (timed or not)
     ~PhaseTimer()
     {
         for (auto e : pool) cudaEventDestroy(e);
@@ -139,6 +141,7 @@ struct PhaseTimer {
     void start(int ph)
     {
         if (!on) return;
+        if (calls[ph]++ % every != 0) return;
         cur = ph;
         cur_a = used;
         cudaEventRecord(ev(), st);
@@ -177,6 +180,7 @@ struct PhaseTimer {
         s.launches_insert = launches[kPhInsert];
         s.launches_scan = launches[kPhScan];
         s.launches_refine = launches[kPhRefine];
+        s.step_launches = calls[kPhPropagate] + calls[kPhScan];
     }
 };
 
@@ -222,7 +226,8 @@ struct Call {
         CU(cudaEventCreate(&ev0));
         CU(cudaEventCreate(&ev1));
         CU(cudaEventRecord(ev0, st));
-        pt.on = o.profile_phases != 0;
+        pt.on = o.profile_phases > 0;
+        pt.every = o.profile_phases > 0 ? (uint64_t)o.profile_phases : 1;
         pt.st = st;
         return CD_OK;
     }
@@ -238,7 +243,8 @@ cd_status validate_scalars(size_t n, double t0, double t1, double dt, double d, 
     if (!is_fin(dt) || !(dt > 0.0)) return fail(CD_EINVAL, "need dt > 0");
     if (!is_fin(d) || !(d > 0.0)) return fail(CD_EINVAL, "need threshold d > 0");
     if (!is_fin(o.v_margin) || o.v_margin < 0.0) return fail(CD_EINVAL, "need v_margin >= 0");
-    if (!(o.cell_factor >= 1.0) || !is_fin(o.cell_factor)) return fail(CD_EINVAL, "need cell_factor >= 1");
+    if (!(o.cell_factor == 0.0 || o.cell_factor >= 1.0) || !is_fin(o.cell_factor))
+        return fail(CD_EINVAL, "need cell_factor = 0 (auto) or >= 1");
     if (o.n_ranks < 1 || o.rank < 0 || o.rank >= o.n_ranks)
         return fail(CD_EINVAL, "need 0 <= rank < n_ranks");
     for (int c = 0; c < 3; ++c)
@@ -277,12 +283,14 @@ struct OrbitSet {
     DBuf<double> rec;
     DBuf<uint8_t> cls;
     DBuf<uint32_t> perm;   // internal -> caller index
+    int64_t n0 = 0;        // class-0 objects (sorted first)
     Orbits view() const
     {
         Orbits O;
         O.rec = rec.p;
         O.cls = cls.p;
         O.n = (int64_t)perm.n;
+        O.n0 = n0;
         return O;
     }
 };
@@ -322,12 +330,19 @@ cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_opti
     CU(idx.alloc(n));
     CU(keyo.alloc(n));
     CU(S.perm.alloc(n));
-    CU(launch_classify(E, (int64_t)n, key.p, idx.p, st, C.lc));
+    DBuf<unsigned long long> n0(st);
+    CU(n0.alloc(1));
+    CU(cudaMemsetAsync(n0.p, 0, sizeof(unsigned long long), st));
+    CU(launch_classify(E, (int64_t)n, key.p, idx.p, n0.p, st, C.lc));
+    unsigned long long hn0 = 0;
+    CU(cudaMemcpyAsync(&hn0, n0.p, sizeof hn0, cudaMemcpyDeviceToHost, st));
     CU(sort_pairs_u32(key.p, keyo.p, idx.p, S.perm.p, n, 3, st, C.lc));
     CU(S.rec.alloc((size_t)kNCol * n));
     CU(S.cls.alloc(n));
     CU(launch_build_records(E, S.perm.p, (int64_t)n, S.rec.p, S.cls.p, st, C.lc));
     C.pt.stop();
+    CU(cudaStreamSynchronize(st));   // hn0 is needed on the host
+    S.n0 = (int64_t)hn0;
     return CD_OK;
 }
 
@@ -339,6 +354,28 @@ uint64_t next_pow2(uint64_t x)
 }
 
 enum class Want { Conj, Cand };
+
+// Cell edge factor m (L = m g_c) from the measured candidate rate c (pairs within g_c per
+// object-step): the expected local density is 2c / (4 pi / 3) objects per g_c^3.  Per object
+// the scan probes (1 + 2/m)^3 - 1 cells (ball mode, m >= 2) or 13 (half-shell, m = 1) and walks
+// the objects of those cells (~ (m + 2)^3 x density, or 27 x density / 2 in half-shell mode);
+// a walked object costs about 1.5 probes.  Only performance depends on m (any L >= g_c gives
+// the same candidate set).
+double choose_cell_factor(double c)
+{
+    const double dens = 2.0 * c / 4.18879;
+    double best = 1.0, bestcost = 13.0 + 1.5 * 13.5 * dens;
+    const double cand[] = {2.0, 3.0, 4.0, 5.0, 6.0, 8.0};
+    for (double m : cand) {
+        const double probes = std::pow(1.0 + 2.0 / m, 3.0) - 1.0;
+        const double cost = probes + 1.5 * std::pow(m + 2.0, 3.0) * dens;
+        if (cost < bestcost) {
+            bestcost = cost;
+            best = m;
+        }
+    }
+    return best;
+}
 
 struct Result {
     DBuf<Conj> conj;        // unsorted conjunction records (internal ids)
@@ -359,7 +396,10 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     stats.steps = (uint64_t)(ke - kb);
     stats.object_steps = (uint64_t)(ke - kb) * (uint64_t)n;
     const double gc = d + o.v_margin * dt;   // Eq. 1
-    double L = gc * o.cell_factor;
+    // grid cell edge L = m g_c (m = cell_factor; 0 = auto: start at 4, then choose from the
+    // candidate density measured in the first round, see choose_cell_factor)
+    const bool auto_cell = o.cell_factor == 0.0;
+    double L = gc * (auto_cell ? 4.0 : o.cell_factor);
     if (L < gc * (1.0 + 1e-12)) L = gc * (1.0 + 1e-12);
     GridGeom g;
     g.ox = o.grid_origin[0];
@@ -380,28 +420,33 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     int64_t Bmax = std::max<int64_t>(1, (int64_t)(target / (size_t)n));
     Bmax = std::min<int64_t>(Bmax, std::min<int64_t>(ke - kb, 65535));
 
-    // per-step grid arena: two ping-pong table sets [slots | occupancy bitmap] x Bmax, then the
-    // entries; batch b builds set b & 1 while its scan zeroes set (b + 1) & 1
+    // per-step grid arena: [slot set 0 | slot set 1 | bitmap set 0 | 1 | 2] x Bmax tables, then
+    // two entry buffers.  Launch i of a round builds batch b+1 (slot set (b+1) % 2 with tag
+    // (b+1) % 126 + 1, bitmap set (b+1) % 3, entries (b+1) % 2), scans batch b and zeroes bitmap set
+    // (b+2) % 3.  Slot sets are zeroed only when their tags wrap.
     const uint64_t nbits = std::max<uint64_t>(next_pow2((uint64_t)n * 32), 1024);   // >= 32 bits/object
     const uint32_t bwords = (uint32_t)(nbits / 32);
     const size_t slot_bytes = sizeof(Slot) * (size_t)Bmax * M;
     const size_t bit_bytes = ((sizeof(uint32_t) * (size_t)Bmax * bwords + 255) / 256) * 256;
-    const size_t set_bytes = slot_bytes + bit_bytes;
     const size_t ent_bytes = sizeof(Entry) * (size_t)Bmax * n;
+    const size_t tab_bytes = 2 * slot_bytes + 3 * bit_bytes;
     DBuf<unsigned char> arena(st);
-    CU(arena.alloc(2 * set_bytes + ent_bytes));
-    CU(cudaMemsetAsync(arena.p, 0, 2 * set_bytes, st));
-    GridTab tabs[2];
-    for (int h = 0; h < 2; ++h) {
-        unsigned char* base = arena.p + h * set_bytes;
-        tabs[h] = GridTab{reinterpret_cast<Slot*>(base), reinterpret_cast<uint32_t*>(base + slot_bytes),
-                          (uint32_t)(nbits - 1), bwords};
-    }
-    Entry* ents = reinterpret_cast<Entry*>(arena.p + 2 * set_bytes);
+    CU(arena.alloc(tab_bytes + 2 * ent_bytes));
+    CU(cudaMemsetAsync(arena.p, 0, tab_bytes, st));
+    Slot* slotset[2] = {reinterpret_cast<Slot*>(arena.p), reinterpret_cast<Slot*>(arena.p + slot_bytes)};
+    uint32_t* bitset[3];
+    for (int h = 0; h < 3; ++h)
+        bitset[h] = reinterpret_cast<uint32_t*>(arena.p + 2 * slot_bytes + h * bit_bytes);
+    Entry* entbuf[2] = {reinterpret_cast<Entry*>(arena.p + tab_bytes),
+                        reinterpret_cast<Entry*>(arena.p + tab_bytes + ent_bytes)};
+    auto tab_of = [&](uint64_t b) {
+        return GridTab{slotset[b % 2], bitset[b % 3], (uint32_t)(nbits - 1), bwords};
+    };
+    auto tag_of = [](uint64_t b) { return (uint32_t)(b % kMaxTag) + 1u; };
     uint64_t batch_no = 0;
-    // persisting-L2 window over the table set being built/scanned (slots + bitmap): these take the
-    // random atomics and probes, while records, entries and the zeroing stream past them
-    L2Win wins[2];
+    // persisting-L2 window over the slot and bitmap sets (they take the random atomics and
+    // probes; records, entries and candidate writes stream past them)
+    L2Win win;
     if (o.l2_persist) {
         int maxwin = 0, maxpersist = 0;
         cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, C.dev);
@@ -409,17 +454,15 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         if (maxwin > 0 && maxpersist > 0) {
             size_t cur = 0;
             cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
-            const size_t setaside = std::min<size_t>((size_t)maxpersist, set_bytes);
+            const size_t setaside = std::min<size_t>((size_t)maxpersist, tab_bytes);
             if (cur < setaside) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside);
             cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
-            for (int h = 0; h < 2; ++h) {
-                wins[h].on = cur > 0;
-                wins[h].w.base_ptr = arena.p + h * set_bytes;
-                wins[h].w.num_bytes = std::min<size_t>(set_bytes, (size_t)maxwin);
-                wins[h].w.hitRatio = (float)std::min(1.0, (double)cur / (double)wins[h].w.num_bytes);
-                wins[h].w.hitProp = cudaAccessPropertyPersisting;
-                wins[h].w.missProp = cudaAccessPropertyStreaming;
-            }
+            win.on = cur > 0;
+            win.w.base_ptr = arena.p;
+            win.w.num_bytes = std::min<size_t>(tab_bytes, (size_t)maxwin);
+            win.w.hitRatio = (float)std::min(1.0, (double)cur / (double)win.w.num_bytes);
+            win.w.hitProp = cudaAccessPropertyPersisting;
+            win.w.missProp = cudaAccessPropertyStreaming;
         }
         cudaGetLastError();   // persistence is best effort
     }
@@ -455,19 +498,47 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         const int64_t Rk = std::min<int64_t>(Rsteps, ke - k);
         CU(cudaMemsetAsync(&ctrl.p->n_cand, 0, sizeof(unsigned long long), st));
         CU(cudaMemsetAsync(nwork.p, 0, sizeof(unsigned long long), st));
-        for (int64_t kk = k; kk < k + Rk; kk += Bmax) {
-            const int B = (int)std::min<int64_t>(Bmax, k + Rk - kk);
-            const GridTab& cur = tabs[batch_no & 1];
-            const GridTab& nxt = tabs[(batch_no + 1) & 1];
-            C.pt.start(kPhPropagate);
-            const L2Win* win = &wins[batch_no & 1];
-            CU(launch_prop_insert(O, g, cur, ents, mask, kk, B, t0, dt, ctrl.p, win, st, C.lc));
-            C.pt.stop();
-            C.pt.start(kPhScan);
-            CU(launch_scan(g, cur, nxt, (int)Bmax, ents, n, mask, kk, kKeyTag, B, q.p, qcap, ctrl.p,
-                           win, st, C.lc));
-            C.pt.stop();
-            ++batch_no;
+        {
+            // software pipeline over the round's batches: launch i builds batch i and scans i - 1
+            const int64_t J = (Rk + Bmax - 1) / Bmax;
+            for (int64_t i = 0; i <= J; ++i) {
+                StepArgs sa{};
+                sa.O = O;
+                sa.g = g;
+                sa.mask = mask;
+                sa.t0 = t0;
+                sa.dt = dt;
+                sa.q = q.p;
+                sa.qcap = qcap;
+                sa.ctrl = ctrl.p;
+                const uint64_t bb = batch_no + (uint64_t)i;   // batch built in this launch
+                if (i < J) {
+                    if (bb % kMaxTag < 2 && bb >= 2) {
+                        // this slot set's tags wrap with this batch: zero it (its last scan, of
+                        // batch bb - 2, finished in the previous launch)
+                        CU(cudaMemsetAsync(slotset[bb % 2], 0, slot_bytes, st));
+                    }
+                    sa.build_k0 = k + i * Bmax;
+                    sa.build_B = std::min<int64_t>(Bmax, k + Rk - sa.build_k0);
+                    sa.build_tab = tab_of(bb);
+                    sa.build_ents = entbuf[bb % 2];
+                    sa.build_tag = tag_of(bb);
+                }
+                if (i > 0) {
+                    sa.scan_k0 = k + (i - 1) * Bmax;
+                    sa.scan_B = std::min<int64_t>(Bmax, k + Rk - sa.scan_k0);
+                    sa.scan_tab = tab_of(bb - 1);
+                    sa.scan_ents = entbuf[(bb - 1) % 2];
+                    sa.scan_tag = tag_of(bb - 1);
+                }
+                sa.zero_bits = bitset[(bb + 1) % 3];   // batch bb - 2's bitmaps, next built by bb + 1
+                sa.zero_bits_words = bwords;
+                sa.zero_depth = Bmax;
+                C.pt.start(i < J && i == 0 ? kPhPropagate : kPhScan);
+                CU(launch_step(sa, &win, st, C.lc));
+                C.pt.stop();
+            }
+            batch_no += (uint64_t)J;
         }
         if (want == Want::Conj) {
             C.pt.start(kPhRefine);
@@ -548,6 +619,13 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             R.n_cand += hctrl->n_cand;
         }
         conj_before = hctrl->n_conj;
+        if (auto_cell && k == kb) {   // first round done: re-pick the cell edge from the density
+            const double m = choose_cell_factor((double)hctrl->n_cand / ((double)Rk * (double)n));
+            L = gc * m;
+            if (L < gc * (1.0 + 1e-12)) L = gc * (1.0 + 1e-12);
+            g.inv_cell = 1.0 / L;
+            g.halfshell = L < 2.0 * gc ? 1 : 0;
+        }
         if (!o.round_steps) {
             const double rate = std::max(1.0, (double)hctrl->n_cand / (double)Rk);
             Rsteps = std::max<int64_t>(1, std::min<int64_t>(1 << 16, (int64_t)(0.5 * qcap / rate)));
@@ -640,8 +718,8 @@ void cd_options_init(cd_options* o)
     o->device = -1;
     o->rank = 0;
     o->n_ranks = 1;
-    o->cell_factor = 1.0;
-    o->l2_persist = 1;
+    o->cell_factor = 0.0;   // auto (1.0 = the paper's cell edge g_c, 27-cell neighbourhood)
+    o->l2_persist = 0;
 }
 
 cd_status cd_screen(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,

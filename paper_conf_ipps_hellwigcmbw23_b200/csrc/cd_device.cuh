@@ -44,6 +44,7 @@ struct Orbits {
     const double* rec;   // kNCol x n
     const uint8_t* cls;  // eccentricity class per object
     int64_t n;
+    int64_t n0;          // objects [0, n0) are class 0 (records sorted by class)
     // records are streamed once per step: evict-first so they do not push the per-step grid
     // (slots, bitmap, entries) out of L2
     __device__ __forceinline__ double at(int c, int64_t r) const { return __ldcs(rec + c * n + r); }
@@ -74,6 +75,33 @@ __device__ __forceinline__ void sincos_small(double d, double& s, double& c)
     pc = fma(pc, x, -1.0 / 24.0);
     pc = fma(pc, x, 0.5);
     c = fma(-pc, x, 1.0);
+}
+
+// sin and cos for the Contour centre c in [-0.5, 2 pi + 0.5] (also correct for |x| < ~1e5):
+// Cody-Waite reduction by pi/2 (two-part constant, fused multiply-adds) and Taylor series on
+// [-pi/4, pi/4] (truncation < 1e-19).  No slow path, few registers.
+__device__ __forceinline__ void sincos_fast(double x, double& s, double& c)
+{
+    const double k = rint(x * 0.63661977236758134308);
+    double r = fma(-k, 1.5707963267948966, x);
+    r = fma(-k, 6.123233995736766e-17, r);
+    double sr, cr;
+    sincos_small(r, sr, cr);
+    const int q = (int)k & 3;
+    s = q == 0 ? sr : q == 1 ? cr : q == 2 ? -sr : -cr;
+    c = q == 0 ? cr : q == 1 ? -sr : q == 2 ? -cr : sr;
+}
+
+// 1/b from the hardware fp64 reciprocal estimate plus two Newton steps (full precision for the
+// finite, non-zero arguments used here; no IEEE-division slow path)
+__device__ __forceinline__ double rcp_fast(double b)
+{
+    double r;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(b));
+    double e = fma(-b, r, 1.0);
+    r = fma(r, e, r);
+    e = fma(-b, r, 1.0);
+    return fma(r, e, r);
 }
 
 // M = (M0 + n t) reduced to [0, 2pi)
@@ -156,7 +184,7 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
     const double dc = lower ? rho : -rho;
     const double c = M + dc;
     double sc, cc;
-    sincos(c, &sc, &cc);
+    sincos_fast(c, sc, cc);
     double ecr, esr;
     if (N == 4) {
         // class 0 (e <= 0.01, rho <= 0.005): the six per-object constants are evaluated here by
@@ -177,9 +205,11 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
     } else if (fp == 0.0) {
         delta = -rho;
     } else {
-        double num = 1.0 / f0 + 1.0 / fp;   // e^{2i*0}=1, e^{2i*pi}=1
-        double den = 1.0 / f0 - 1.0 / fp;   // e^{i*0}=1,  e^{i*pi}=-1
-#pragma unroll
+        const double i0 = rcp_fast(f0);
+        const double ip = rcp_fast(fp);
+        double num = i0 + ip;   // e^{2i*0}=1, e^{2i*pi}=1
+        double den = i0 - ip;   // e^{i*0}=1,  e^{i*pi}=-1
+#pragma unroll(N == 4 ? 1 : 1)
         for (int j = 1; j <= (N - 2) / 2; ++j) {
             constexpr int cl = N == 4 ? 0 : N == 6 ? 1 : N == 8 ? 2 : N == 12 ? 3 : 4;
             const double ct = kNodes[cl][j - 1][0], st = kNodes[cl][j - 1][1];
@@ -205,66 +235,60 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
             const double ima = fma(rho, st, -ecos_a * sh);
             const double reb = fma(-rho, ct, dc) - esin_b * ch;
             const double imb = fma(rho, st, -ecos_b * sh);
-            const double ia = 2.0 / fma(rea, rea, ima * ima);
-            const double ib = 2.0 / fma(reb, reb, imb * imb);
+            const double ia = 2.0 * rcp_fast(fma(rea, rea, ima * ima));
+            const double ib = 2.0 * rcp_fast(fma(reb, reb, imb * imb));
             // th_b = pi - th: cos th_b = -ct, sin th_b = st, cos 2th_b = c2t, sin 2th_b = -s2t
             num += ia * fma(c2t, rea, s2t * ima) + ib * fma(c2t, reb, -s2t * imb);
             den += ia * fma(ct, rea, st * ima) + ib * fma(-ct, reb, st * imb);
         }
-        delta = rho * (num / den);
+        delta = rho * (num * rcp_fast(den));
     }
     E = c + delta;
     double sd, cd;
-    sincos_small(delta, sd, cd);
+    if (N == 4) {   // |delta| <= rho <= 0.005: truncation < 1e-24
+        const double x = delta * delta;
+        sd = delta * fma(fma(fma(-1.0 / 5040.0, x, 1.0 / 120.0), x, -1.0 / 6.0), x, 1.0);
+        cd = fma(fma(fma(-1.0 / 720.0, x, 1.0 / 24.0), x, -0.5), x, 1.0);
+    } else {
+        sincos_small(delta, sd, cd);
+    }
     sE = fma(sc, cd, cc * sd);
     cE = fma(cc, cd, -sc * sd);
 }
 
-// Classes 1-4 (e > 0.01, a small minority of the LEO-heavy populations) live out of line so
-// the register allocation of the hot class-0 path (N = 4) stays small.
-static __device__ __noinline__ void kepler_solve_slow(double M, double e, int cls, Orbits O, int64_t r,
-                                               double* E, double* sE, double* cE)
-{
-    switch (cls) {
-    case 1: contour_core<6>(M, e, O, r, *E, *sE, *cE); break;
-    case 2: contour_core<8>(M, e, O, r, *E, *sE, *cE); break;
-    case 3: contour_core<12>(M, e, O, r, *E, *sE, *cE); break;
-    default: {
-        contour_core<16>(M, e, O, r, *E, *sE, *cE);
-        // e > 0.6: Newton polish of the contour estimate (R15)
-        for (int it = 0; it < 8; ++it) {
-            const double dE = (*E - e * *sE - M) / (1.0 - e * *cE);
-            *E -= dE;
-            sincos(*E, sE, cE);
-            if (fabs(dE) <= 1e-15 * fmax(1.0, fabs(*E))) break;
-        }
-    }
-    }
-}
-
+// Eccentricity-class dispatch (objects are sorted by class, so warps are uniform).
 __device__ __forceinline__ void kepler_solve(double M, double e, int cls, const Orbits& O,
                                              int64_t r, double& E, double& sE, double& cE)
 {
-    if (cls == 0) {
-        contour_core<4>(M, e, O, r, E, sE, cE);
-    } else {
-        double e_, s_, c_;
-        kepler_solve_slow(M, e, cls, O, r, &e_, &s_, &c_);
-        E = e_;
-        sE = s_;
-        cE = c_;
+    switch (cls) {
+    case 0: contour_core<4>(M, e, O, r, E, sE, cE); break;
+    case 1: contour_core<6>(M, e, O, r, E, sE, cE); break;
+    case 2: contour_core<8>(M, e, O, r, E, sE, cE); break;
+    case 3: contour_core<12>(M, e, O, r, E, sE, cE); break;
+    default:
+        contour_core<16>(M, e, O, r, E, sE, cE);
+        if (e > 0.8) {   // Newton polish of the contour estimate (R15)
+            for (int it = 0; it < 8; ++it) {
+                const double dE = (E - e * sE - M) * rcp_fast(1.0 - e * cE);
+                E -= dE;
+                sincos_fast(E, sE, cE);
+                if (fabs(dE) <= 1e-15 * fmax(1.0, fabs(E))) break;
+            }
+        }
     }
 }
 
 // Position (and velocity) of object r at time t.
 //   r = (cos E - e) aP + sin E bQ;     v = n/(1 - e cos E) (-sin E aP + cos E bQ)
-template <bool kVel>
+// kClass: 0 = object known to be class 0 (lean path), -1 = any class
+template <bool kVel, int kClass = -1>
 __device__ __forceinline__ void state(const Orbits& O, int64_t r, double t, double p[3], double v[3])
 {
     const double e = O.at(kE, r);
     const double M = mean_anomaly(O.at(kM0, r), O.at(kNm, r), t);
     double E, sE, cE;
-    kepler_solve(M, e, O.cls[r], O, r, E, sE, cE);
+    if (kClass == 0) contour_core<4>(M, e, O, r, E, sE, cE);
+    else kepler_solve(M, e, O.cls[r], O, r, E, sE, cE);
     const double x = cE - e;
     const double ap[3] = {O.at(kAPx, r), O.at(kAPy, r), O.at(kAPz, r)};
     const double bq[3] = {O.at(kBQx, r), O.at(kBQy, r), O.at(kBQz, r)};
@@ -281,12 +305,14 @@ __device__ __forceinline__ void state(const Orbits& O, int64_t r, double t, doub
 // grid cells and keys ("calculates the grid cell based on the Cartesian coordinates")
 // ---------------------------------------------------------------------------------------
 // Cell keys pack 19 bits per axis (cells in [-(2^18 - 2), 2^18 - 2], i.e. +-262,142 cells of
-// edge L >= g_c: +-46,000 km at g_c = 0.18 km); the top 7 bits of a stored key word hold a
-// non-zero tag so a stored key is never the all-zero empty value.
+// edge L >= g_c: +-46,000 km at g_c = 0.18 km); the top 7 bits of a stored key word hold the tag
+// (1..126) of the build pass that wrote it.  A slot whose tag differs from the current pass is
+// empty (P:147 reserves a value for "empty"; tagging lets a table be reused without clearing it
+// every step -- tables are zeroed only when the tags wrap).
 constexpr int64_t kKeyBias = int64_t(1) << 18;
 constexpr int64_t kCellMax = kKeyBias - 2;   // valid cells in [-kCellMax, kCellMax]
 constexpr int kTagShift = 57;
-constexpr uint32_t kKeyTag = 1;
+constexpr uint32_t kMaxTag = 126;
 constexpr uint32_t kNil = 0xffffffffu;
 
 __device__ __forceinline__ uint64_t pack_key(int64_t cx, int64_t cy, int64_t cz)
@@ -359,27 +385,28 @@ __device__ __forceinline__ bool cas128(Slot* s, unsigned long long& e0, unsigned
     return ok;
 }
 
-// Non-blocking insert of object r into the cell `key`.  Tables are zeroed before
-// each use, so the first attempt on a slot is a blind CAS against the empty value {0, 0}: claiming
-// an empty cell costs one atomic; a slot already holding the key pushes r onto its list (CAS of
-// the head); a slot of another cell moves on along the probe sequence (Eq. 2).  Returns the
-// previous list head (r's `next`), kNil if r is the first object of its cell.
+// Non-blocking insert of object r into the cell `key`.  A slot whose key word carries
+// another pass's tag is empty: it is claimed by a 128-bit CAS against the value just read; a slot
+// already holding the key (this pass) pushes r onto its list (CAS of the head); a slot of another
+// cell moves on along the probe sequence (Eq. 2).  Returns the previous list head (r's `next`),
+// kNil if r is the first object of its cell.
 __device__ __forceinline__ uint32_t grid_insert(Slot* slots, uint64_t mask, unsigned long long key,
                                                 uint32_t tag, uint32_t r)
 {
     const unsigned long long tk = key | ((unsigned long long)tag << kTagShift);
     uint64_t h = fmix64(key) & mask;
-    unsigned long long e0 = 0ull, e1 = 0ull;
     while (true) {
-        if (cas128(slots + h, e0, e1, tk, (unsigned long long)r))
-            return e0 == 0ull ? kNil : (uint32_t)e1;
-        // failed: (e0, e1) = current contents
-        if (e0 != tk) {   // another cell (the slot cannot return to empty): next slot
-            h = (h + 1) & mask;
-            e0 = 0ull;
-            e1 = 0ull;
+        unsigned long long w0, w1;
+        asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(w0), "=l"(w1) : "l"(slots + h));
+        while (true) {
+            const bool stale = (uint32_t)(w0 >> kTagShift) != tag;
+            if (!stale && w0 != tk) break;   // another cell of this pass: next slot
+            const unsigned long long prev = w1;
+            if (cas128(slots + h, w0, w1, tk, (unsigned long long)r))
+                return stale ? kNil : (uint32_t)prev;
+            // lost a race: (w0, w1) now hold the slot's current contents; re-evaluate
         }
-        // same cell: retry the push with the observed head
+        h = (h + 1) & mask;
     }
 }
 

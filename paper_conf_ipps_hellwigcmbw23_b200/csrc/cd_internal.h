@@ -41,7 +41,7 @@ struct RefineParams {
 
 // ---- precompute (a1) -------------------------------------------------------------------
 cudaError_t launch_classify(const Elements& el, int64_t n, uint32_t* key, uint32_t* idx,
-                            cudaStream_t st, LaunchCount& lc);
+                            unsigned long long* n0, cudaStream_t st, LaunchCount& lc);
 cudaError_t launch_build_records(const Elements& el, const uint32_t* perm, int64_t n,
                                  double* rec, uint8_t* cls, cudaStream_t st, LaunchCount& lc);
 cudaError_t launch_propagate_out(const cdk::Orbits& O, const uint32_t* perm, const double* t,
@@ -51,16 +51,32 @@ cudaError_t launch_propagate_out(const cdk::Orbits& O, const uint32_t* perm, con
 // ---- grid build + scan (a2-a6) ---------------------------------------------------------
 cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long long v,
                             cudaStream_t st, LaunchCount& lc);
-// Fused propagate + cell key + insert; the tables of `tab` must be zero on entry.
-cudaError_t launch_prop_insert(const cdk::Orbits& O, const cdk::GridGeom& g, const cdk::GridTab& tab,
-                               cdk::Entry* ents, uint64_t mask, int64_t k0, int B, double t0,
-                               double dt, cdk::Ctrl* ctrl, const L2Win* win, cudaStream_t st,
-                               LaunchCount& lc);
-// Neighbour scan of the batch in `tab`; also zeroes the ping-pong set `clr` for the next batch.
-cudaError_t launch_scan(const cdk::GridGeom& g, const cdk::GridTab& tab, const cdk::GridTab& clr,
-                        int nclr, const cdk::Entry* ents, int64_t n, uint64_t mask, int64_t k0, uint32_t tag,
-                        int B, cdk::Cand* q, size_t qcap, cdk::Ctrl* ctrl, const L2Win* win,
-                        cudaStream_t st, LaunchCount& lc);
+// One batch launch of the fused step kernel: build batch b+1 into build_tab (slots tagged
+// build_tag, bitmap zero on entry), scan batch b in scan_tab (tag scan_tag), zero the bitmap set
+// zero_bits (zero_depth tables) for batch b+2.
+struct StepArgs {
+    cdk::Orbits O;
+    cdk::GridGeom g;
+    uint64_t mask;
+    double t0, dt;
+    int64_t build_B, build_k0;   // build_B = 0: no build role
+    cdk::GridTab build_tab;
+    cdk::Entry* build_ents;
+    uint32_t build_tag;
+    int64_t scan_B, scan_k0;     // scan_B = 0: no scan role
+    cdk::GridTab scan_tab;
+    const cdk::Entry* scan_ents;
+    uint32_t scan_tag;
+    uint32_t* zero_bits;
+    int64_t zero_bits_words;     // words per table
+    int64_t zero_depth;          // tables to zero (0: none)
+    cdk::Cand* q;
+    size_t qcap;
+    cdk::Ctrl* ctrl;
+    int64_t nbA, nbB, nbC;       // blocks per step of roles A, B, C (filled by launch_step)
+    int64_t nCblocks;            // role-C blocks in the launch
+};
+cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCount& lc);
 
 // ---- refinement (a7) -------------------------------------------------------------------
 cudaError_t launch_prefilter(const cdk::Orbits& O, const RefineParams& p, const cdk::Cand* q,

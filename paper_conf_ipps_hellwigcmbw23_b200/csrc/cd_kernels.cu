@@ -52,15 +52,24 @@ __device__ __forceinline__ void append(T* buf, size_t cap, unsigned long long* c
     if (idx < cap) buf[idx] = v;
 }
 
+__device__ __forceinline__ void append_count(unsigned long long* cnt)
+{
+    cg::coalesced_group g = cg::coalesced_threads();
+    if (g.thread_rank() == 0) atomicAdd(cnt, (unsigned long long)g.size());
+}
+
 // ---------------------------------------------------------------------------------------
 // a1: per-object precompute
 // ---------------------------------------------------------------------------------------
-__global__ void k_classify(Elements el, int64_t n, uint32_t* key, uint32_t* idx)
+__global__ void k_classify(Elements el, int64_t n, uint32_t* key, uint32_t* idx,
+                           unsigned long long* n0)
 {
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i >= n) return;
-    key[i] = (uint32_t)ecc_class(el.e[i]);
+    const int cl = ecc_class(el.e[i]);
+    key[i] = (uint32_t)cl;
     idx[i] = (uint32_t)i;
+    if (cl == 0) append_count(n0);
 }
 
 __global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, int64_t n,
@@ -124,9 +133,9 @@ __global__ void k_propagate_out(Orbits O, const uint32_t* __restrict__ perm,
 }
 
 cudaError_t launch_classify(const Elements& el, int64_t n, uint32_t* key, uint32_t* idx,
-                            cudaStream_t st, LaunchCount& lc)
+                            unsigned long long* n0, cudaStream_t st, LaunchCount& lc)
 {
-    k_classify<<<blocks_for(n, 256), 256, 0, st>>>(el, n, key, idx);
+    k_classify<<<blocks_for(n, 256), 256, 0, st>>>(el, n, key, idx, n0);
     lc.bump();
     return cudaGetLastError();
 }
@@ -175,28 +184,26 @@ cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long l
 }
 
 // ---------------------------------------------------------------------------------------
-// a2-a4: one thread per (object, step) ("one thread per tuple"): Contour Kepler solve and
-// Cartesian position, cell key, non-blocking insert into the step's hash grid (P:135-150,
-// Eq. 2) and its occupancy bitmap; the entry {x, y, z, next} (Fig. 6) is written once,
-// coalesced.
+// a2-a4: build -- one thread per (object, step) ("one thread per tuple"): Contour Kepler
+// solve and Cartesian position, cell key, non-blocking insert into the step's hash grid
+// (Eq. 2) and its occupancy bitmap; the entry {x, y, z, next} (Fig. 6) is
+// written once, coalesced.  kClass0: objects [0, n0) (e <= 0.01: lean N = 4 Contour path).
 // ---------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(256, 4) k_prop_insert(Orbits O, GridGeom g, GridTab tab,
-                                                        Entry* __restrict__ ents, uint64_t mask,
-                                                        int64_t k0, double t0, double dt, Ctrl* ctrl)
+template <bool kClass0>
+__device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, const GridTab& tab,
+                                         Entry* __restrict__ ents, uint64_t mask, int64_t k0, int s,
+                                         int64_t r, double t0, double dt, uint32_t tag, Ctrl* ctrl)
 {
-    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (r >= O.n) return;
-    const int s = blockIdx.y;
     const double t = fma((double)(k0 + s), dt, t0);
     double p[3], v[3];
-    state<false>(O, r, t, p, v);
+    state<false, kClass0 ? 0 : -1>(O, r, t, p, v);
     int64_t c[3];
     uint32_t next = kNil;
     if (cell_of(g, p, c)) {
         const unsigned long long key = pack_key(c[0], c[1], c[2]);
         const uint32_t hb = bit_of(key) & tab.bmask;
         atomicOr(tab.bits + (size_t)s * tab.bwords + (hb >> 5), 1u << (hb & 31));
-        next = grid_insert(tab.slots + (size_t)s * (mask + 1), mask, key, kKeyTag, (uint32_t)r);
+        next = grid_insert(tab.slots + (size_t)s * (mask + 1), mask, key, tag, (uint32_t)r);
     } else {
         ctrl->err_range = 1;
     }
@@ -216,8 +223,8 @@ __global__ void __launch_bounds__(256, 4) k_prop_insert(Orbits O, GridGeom g, Gr
 //  (2) other cells: half-shell mode (L < 2 g_c, the paper's cell g_c) probes the 13
 //      positive half-shell neighbours -- each unordered pair of cells of a 3x3x3 block once;
 //      ball mode (L >= 2 g_c) probes the 0-7 other cells overlapping |x - p| < g_c -- a pair is
-//      seen from both objects and reported by the smaller index.  The first slot of every probe
-//      is loaded before any is resolved, so a thread's probes overlap in flight.
+//      seen from both objects and reported by the smaller index.  Each probe first tests the
+//      occupancy bitmap (all bitmap loads of a thread are issued together).
 // A pair is a candidate iff |r_i - r_j| < g_c (reading R6); candidates are appended with one
 // atomic per group of converged lanes (P:95 saves ids + sampling step).
 // ---------------------------------------------------------------------------------------
@@ -277,27 +284,11 @@ __device__ __forceinline__ void probe_group(const GridGeom& g, const Slot* __res
     }
 }
 
-__global__ void __launch_bounds__(256, 1) k_scan(GridGeom g, GridTab tab, GridTab clr, int nclr,
-                                                 const Entry* __restrict__ ents, int64_t n,
-                                                 uint64_t mask, int64_t k0, uint32_t tag,
-                                                 Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
+__device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
+                                        const Entry* __restrict__ ents, int64_t n, uint64_t mask,
+                                        int64_t k0, int s, int64_t r, uint32_t tag,
+                                        Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
 {
-    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    const int s = blockIdx.y;
-    // side job: zero the other (ping-pong) table set for the next batch -- tables s, s + B, ...
-    // below nclr (the allocated batch depth), so a deeper next batch also finds zeroed tables
-    {
-        const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-        const int64_t nth = (int64_t)gridDim.x * blockDim.x;
-        for (int ss = s; ss < nclr; ss += (int)gridDim.y) {
-            // streaming stores (evict-first): the zeroed set is not touched until the next batch
-            ulonglong2* cs = reinterpret_cast<ulonglong2*>(clr.slots + (size_t)ss * (mask + 1));
-            for (int64_t i = tid; i <= (int64_t)mask; i += nth) __stcs(cs + i, make_ulonglong2(0ull, 0ull));
-            uint4* cb = reinterpret_cast<uint4*>(clr.bits + (size_t)ss * clr.bwords);
-            for (int64_t i = tid; i < (int64_t)(clr.bwords / 4); i += nth) __stcs(cb + i, make_uint4(0u, 0u, 0u, 0u));
-        }
-    }
-    if (r >= n) return;
     const Slot* slots = tab.slots + (size_t)s * (mask + 1);
     const uint32_t* bits = tab.bits + (size_t)s * tab.bwords;
     const Entry* E = ents + (size_t)s * n;
@@ -336,24 +327,62 @@ __global__ void __launch_bounds__(256, 1) k_scan(GridGeom g, GridTab tab, GridTa
     }
 }
 
-cudaError_t launch_prop_insert(const Orbits& O, const GridGeom& g, const GridTab& tab, Entry* ents,
-                               uint64_t mask, int64_t k0, int B, double t0, double dt, Ctrl* ctrl,
-                               const L2Win* win, cudaStream_t st, LaunchCount& lc)
+// ---------------------------------------------------------------------------------------
+// One launch per batch (horizontal fusion): blocks of three roles run side by side, so the
+// latency-bound build (fp64 Contour + atomics) and scan (probes) hide each other's stalls.
+//   role A: build batch b + 1, class-0 objects     (slot set (b+1) % 2, bitmap set (b+1) % 3)
+//   role B: build batch b + 1, objects of classes 1-4
+//   role C: scan batch b (slot set b % 2, bitmap set b % 3), and zero bitmap set (b+2) % 3
+//           (used by batch b - 1, next built by batch b + 2)
+// ---------------------------------------------------------------------------------------
+#ifndef CD_STEP_MINB
+#define CD_STEP_MINB 6
+#endif
+__global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
 {
-    dim3 grid(blocks_for(O.n, 256), (unsigned)B);
-    lc.bump();
-    return launch_ex(k_prop_insert, grid, dim3(256), st, win, O, g, tab, ents, mask, k0, t0, dt, ctrl);
+    const int64_t bx = blockIdx.x;
+    const int64_t nA = a.build_B * a.nbA, nB = a.build_B * a.nbB;
+    if (bx < nA) {
+        const int s = (int)(bx / a.nbA);
+        const int64_t r = (bx % a.nbA) * 256 + threadIdx.x;
+        if (r < a.O.n0)
+            do_build<true>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0, a.dt,
+                           a.build_tag, a.ctrl);
+    } else if (bx < nA + nB) {
+        const int64_t b2 = bx - nA;
+        const int s = (int)(b2 / a.nbB);
+        const int64_t r = a.O.n0 + (b2 % a.nbB) * 256 + threadIdx.x;
+        if (r < a.O.n)
+            do_build<false>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0, a.dt,
+                            a.build_tag, a.ctrl);
+    } else {
+        const int64_t b3 = bx - nA - nB;
+        // zero the bitmap set of batch b + 2 (all Bmax tables), grid-stride over role-C threads
+        const int64_t tid = b3 * 256 + threadIdx.x;
+        const int64_t nth = a.nCblocks * 256;
+        const int64_t nw4 = (int64_t)a.zero_depth * a.zero_bits_words / 4;
+        uint4* zb = reinterpret_cast<uint4*>(a.zero_bits);
+        for (int64_t i = tid; i < nw4; i += nth) zb[i] = make_uint4(0u, 0u, 0u, 0u);
+        if (a.scan_B == 0) return;
+        const int s = (int)(b3 / a.nbC);
+        const int64_t r = (b3 % a.nbC) * 256 + threadIdx.x;
+        if (r < a.O.n)
+            do_scan(a.g, a.scan_tab, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r, a.scan_tag, a.q,
+                    a.qcap, a.ctrl);
+    }
 }
 
-cudaError_t launch_scan(const GridGeom& g, const GridTab& tab, const GridTab& clr, int nclr,
-                        const Entry* ents, int64_t n, uint64_t mask, int64_t k0, uint32_t tag, int B,
-                        Cand* q, size_t qcap, Ctrl* ctrl, const L2Win* win, cudaStream_t st,
-                        LaunchCount& lc)
+cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCount& lc)
 {
-    dim3 grid(blocks_for(n, 256), (unsigned)B);
+    a.nbA = (int64_t)blocks_for(a.O.n0, 256);
+    a.nbB = (int64_t)blocks_for(a.O.n - a.O.n0, 256);
+    a.nbC = (int64_t)blocks_for(a.O.n, 256);
+    a.nCblocks = a.scan_B * a.nbC;
+    if (a.nCblocks == 0 && a.zero_depth > 0) a.nCblocks = 148 * 4;   // zero-only role-C blocks
+    const int64_t blocks = a.build_B * (a.nbA + a.nbB) + a.nCblocks;
+    if (blocks == 0) return cudaSuccess;
     lc.bump();
-    return launch_ex(k_scan, grid, dim3(256), st, win, g, tab, clr, nclr, ents, n, mask, k0, tag, q,
-                     qcap, ctrl);
+    return launch_ex(k_step, dim3((unsigned)blocks), dim3(256), st, win, a);
 }
 
 // ---------------------------------------------------------------------------------------

@@ -48,7 +48,7 @@ def test_version_status_options(cds):
     assert cds.status_str(cds.CD_ENODEV) == "CD_ENODEV"
     o = cds.cd_options()
     cds.cd_options_init(o)
-    assert o.v_margin == 7.8 and o.n_ranks == 1 and o.cell_factor == 1.0 and o.device == -1
+    assert o.v_margin == 7.8 and o.n_ranks == 1 and o.cell_factor == 0.0 and o.device == -1
 
 
 def test_struct_layouts(cds):

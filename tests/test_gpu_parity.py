@@ -95,7 +95,8 @@ def test_candidates_ragged_sizes(n, steps, d):
     assert len(Ko) > 0
 
 
-@pytest.mark.parametrize("kw", [dict(grid_origin=(1234.5, -987.25, 55.125)), dict(cell_factor=2.0),
+@pytest.mark.parametrize("kw", [dict(grid_origin=(1234.5, -987.25, 55.125)), dict(cell_factor=1.0),
+                                dict(cell_factor=2.0), dict(cell_factor=1.5, grid_origin=(-3e3, 7.5, 1e4)),
                                 dict(cell_factor=3.7), dict(batch_object_steps=1),
                                 dict(round_steps=7), dict(batch_object_steps=10 ** 7)])
 def test_candidates_invariance(kw):
