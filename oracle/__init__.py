@@ -23,6 +23,7 @@ SOURCES = sorted(HERE.glob("*.c"))
 MULTI = 1
 DEGENERATE = 2
 COPLANAR = 4
+H_AP, H_COPLANAR, H_PATH, H_TIME = 1, 2, 4, 8
 
 CAND_DTYPE = np.dtype([("i", "<u4"), ("j", "<u4"), ("step", "<u4")])
 CONJ_DTYPE = np.dtype([("i", "<u4"), ("j", "<u4"), ("step", "<u4"), ("flags", "<u4"),
@@ -97,8 +98,8 @@ def _bind_hybrid(L):
                              C.c_double, C.c_double, C.c_int64, C.c_int64, P(C.c_void_p),
                              P(C.c_int64)]
     L.orc_pair_filter.restype = C.c_int
-    L.orc_pair_filter.argtypes = [P(_Elements), C.c_int64, C.c_int64, C.c_double,
-                                  P(C.c_double), P(C.c_int)]
+    L.orc_pair_filter.argtypes = [P(_Elements), C.c_int64, C.c_int64, C.c_double, C.c_double,
+                                  C.c_double, P(C.c_double), C.c_int, P(C.c_int)]
 
 
 def _f64(x):
@@ -203,6 +204,28 @@ def pair_distance(pop, i, j, times):
     g = np.zeros(t.size)
     lib().orc_pair_distance(P.ref, int(i), int(j), _dp(t), t.size, _dp(D), _dp(g))
     return D, g
+
+
+def pair_filter(pop, i, j, d, tlo, thi):
+    """Hybrid filter chain for one pair over [tlo, thi]: (flags, [(lo, hi), ...])."""
+    P = _Pop(pop)
+    iv = np.zeros(64)
+    niv = C.c_int()
+    f = lib().orc_pair_filter(P.ref, int(i), int(j), float(d), float(tlo), float(thi), _dp(iv), 32,
+                              C.byref(niv))
+    return int(f), [(iv[2 * q], iv[2 * q + 1]) for q in range(niv.value)]
+
+
+def hybrid(pop, t0, t1, dt, d, v_margin=7.8, k_begin=0, k_end=-1):
+    """Hybrid variant end to end (O4): conjunctions and the filter-stage counts
+    (candidates, ap_rejected, coplanar, path_rejected, time_rejected, time_window_work)."""
+    P = _Pop(pop)
+    gc = cell_size(d, dt, v_margin)
+    out = C.c_void_p()
+    counts = (C.c_int64 * 6)()
+    c = lib().orc_hybrid(P.ref, P.n, t0, t1, dt, d, gc, k_begin, k_end, C.byref(out), counts)
+    keys = ("candidates", "ap_rejected", "coplanar", "path_rejected", "time_rejected", "window_work")
+    return _take(out, c, CONJ_DTYPE), dict(zip(keys, list(counts)))
 
 
 def cell_size(d, dt, v_margin=7.8):

@@ -15,6 +15,8 @@ typedef struct {
 typedef struct { uint32_t i, j, step; } orc_candidate;
 
 enum { ORC_MULTI = 1u, ORC_DEGENERATE = 2u, ORC_COPLANAR = 4u };
+/* hybrid filter outcomes (orc_pair_filter) */
+enum { ORC_H_AP = 1, ORC_H_COPLANAR = 2, ORC_H_PATH = 4, ORC_H_TIME = 8 };
 
 typedef struct {
     uint32_t i, j, step, flags;
@@ -39,6 +41,10 @@ void    orc_pair_distance(const orc_elements* el, int64_t i, int64_t j, const do
                           double* D, double* g);
 void    orc_candidate_flags(const orc_elements* el, int64_t n, double t0, double dt, double gc,
                             const orc_candidate* cand, int64_t ncand, uint32_t* flags);
+int     orc_pair_filter(const orc_elements* el, int64_t i, int64_t j, double d, double tlo,
+                        double thi, double* iv, int cap, int* niv);
+int64_t orc_hybrid(const orc_elements* el, int64_t n, double t0, double t1, double dt, double d,
+                   double gc, int64_t k_begin, int64_t k_end, void** out, int64_t* counts);
 void    orc_free(void* p);
 
 #ifdef __cplusplus

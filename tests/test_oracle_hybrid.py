@@ -1,0 +1,120 @@
+"""Pins for the hybrid-variant oracle (O4, oracle/cd_oracle_hybrid.c) -- -m "not gpu".
+
+* conservativeness: the filter chain never removes a conjunction that the unfiltered level O3
+  finds on the same coarse candidates (so a filter that rejects true encounters fails);
+* selectivity, per filter, on constructed geometries with a known answer;
+* cross-variant: the hybrid at 9 s and the grid at 1 s find the same encounters (P:318 reports
+  the two variants agree to ~0.1 %), modulo the parity exclusions."""
+import math
+
+import numpy as np
+import pytest
+
+from tools import popgen
+
+MU = 398600.4418
+
+
+def _circ(r, inc, raan, u0, e=0.0, argp=0.0):
+    return (r, e, inc, raan, argp, (u0 - argp) % (2 * math.pi))
+
+
+def _pop(rows):
+    arr = np.array(rows, dtype=np.float64)
+    return {k: np.ascontiguousarray(arr[:, c]) for c, k in enumerate(popgen.FIELDS)}
+
+
+def test_conservative_against_unfiltered(orc):
+    pop, cfg, _ = popgen.make_config(2, n=20000)
+    dt, d = 9.0, 5.0
+    gc = orc.cell_size(d, dt)
+    K = orc.candidates_grid(pop, 0.0, 5400.0, dt, gc)
+    full = orc.conjunctions(pop, 0.0, 5400.0, dt, d, gc, K)
+    hyb, counts = orc.hybrid(pop, 0.0, 5400.0, dt, d)
+    assert counts["candidates"] == len(K)
+    assert counts["ap_rejected"] + counts["path_rejected"] + counts["time_rejected"] > 0.5 * len(K)
+    keep = (full["flags"] & orc.DEGENERATE) == 0
+    a = set(zip(full["i"][keep].tolist(), full["j"][keep].tolist(), full["step"][keep].tolist()))
+    b = set(zip(hyb["i"].tolist(), hyb["j"].tolist(), hyb["step"].tolist()))
+    assert len(a) > 20
+    assert a == b
+    # same minima (TCA, PCA) as the unfiltered search
+    fk = {(int(r["i"]), int(r["j"]), int(r["step"])): r for r in full[keep]}
+    for r in hyb:
+        f = fk[(int(r["i"]), int(r["j"]), int(r["step"]))]
+        assert abs(f["tca"] - r["tca"]) < 1e-6 and abs(f["pca"] - r["pca"]) < 1e-9
+
+
+def test_ap_filter_disjoint_shells(orc):
+    pop = _pop([_circ(7000.0, 0.5, 0.0, 0.0), _circ(7100.0, 1.2, 1.0, 0.0)])
+    f, _ = orc.pair_filter(pop, 0, 1, 2.0, 0.0, 6000.0)
+    assert f == orc.H_AP
+    pop = _pop([_circ(7000.0, 0.5, 0.0, 0.0), _circ(7001.5, 1.2, 1.0, 0.0)])
+    assert orc.pair_filter(pop, 0, 1, 2.0, 0.0, 6000.0)[0] != orc.H_AP
+
+
+def test_coplanar_pair(orc):
+    pop = _pop([_circ(7000.0, 0.9, 0.3, 0.0), _circ(7000.5, 0.9, 0.3, 1.0)])
+    assert orc.pair_filter(pop, 0, 1, 2.0, 0.0, 6000.0)[0] == orc.H_COPLANAR
+    # tiny mutual inclination: d / (q sin D) >= 1 -> still coplanar
+    pop = _pop([_circ(7000.0, 0.9, 0.3, 0.0), _circ(7000.5, 0.9 + 1e-4, 0.3, 1.0)])
+    assert orc.pair_filter(pop, 0, 1, 2.0, 0.0, 6000.0)[0] == orc.H_COPLANAR
+
+
+def test_time_windows_case_a(orc):
+    """Closed-form case A: common node, both at the node at t_node -> the time
+    windows contain the closed-form TCA; shift B's phase by a quarter orbit -> time-excluded."""
+    r, delta, u0 = 7000.0, 1.0, 0.3
+    n = math.sqrt(MU / r ** 3)
+    phi = 2 * math.asin(1.0 / (2 * r * math.cos(delta / 2)))    # PCA = 1 km
+    pop = _pop([_circ(r, 0.4, 0.7, -u0), _circ(r, 0.4 + delta, 0.7, -u0 + phi)])
+    tca = (u0 - phi / 2) / n
+    f, iv = orc.pair_filter(pop, 0, 1, 2.0, tca - 20.0, tca + 20.0)
+    assert f == 0 and iv
+    assert any(lo <= tca <= hi for lo, hi in iv)
+    # B a quarter orbit behind: never near the node when A is
+    pop2 = _pop([_circ(r, 0.4, 0.7, -u0), _circ(r, 0.4 + delta, 0.7, -u0 + math.pi / 2)])
+    f2, iv2 = orc.pair_filter(pop2, 0, 1, 2.0, tca - 20.0, tca + 20.0)
+    assert f2 == orc.H_TIME and not iv2
+
+
+def test_orbit_path_filter(orc):
+    """Eccentric orbits crossing at a node where their radii differ by more than d at both nodes:
+    perigee 6900 x apogee 7500 vs circular 7300 km in a plane whose node is at the first
+    orbit's perigee/apogee line -> radial gap 400 / 200 km at the two nodes."""
+    a1, e1 = 7200.0, 300.0 / 7200.0
+    pop = _pop([(a1, e1, 0.5, 0.0, 0.0, 0.0), _circ(7300.0, 1.3, 0.0, 0.0)])
+    f, _ = orc.pair_filter(pop, 0, 1, 2.0, 0.0, 20000.0)
+    assert f == orc.H_PATH
+    # same geometry with the circular orbit at 7500 km: the apogee node is open
+    pop = _pop([(a1, e1, 0.5, 0.0, 0.0, 0.0), _circ(7500.0, 1.3, 0.0, 0.0)])
+    assert orc.pair_filter(pop, 0, 1, 2.0, 0.0, 20000.0)[0] in (0, orc.H_TIME)
+
+
+def test_hybrid_agrees_with_grid(orc):
+    """the grid and hybrid variants find the same encounters (up to ~0.1 %).  Here:
+    every hybrid (9 s) conjunction is a grid (1 s) conjunction with the same TCA and vice versa,
+    except encounters faster than 2 x 7.8 km/s (Eq. 1's assumption, R18) and the exclusions."""
+    pop, cfg, _ = popgen.make_config(2, n=20000)
+    d, t1 = 2.0, 3600.0
+    hyb, _ = orc.hybrid(pop, 0.0, t1, 9.0, d)
+    K, grid = orc.screen_grid(pop, 0.0, t1, 1.0, d)
+
+    def keyset(a, dt):
+        out = {}
+        for r in a:
+            if r["flags"] & orc.DEGENERATE:
+                continue
+            if abs(r["pca"] - d) < 1e-6 or r["tca"] < 1e-3 or r["tca"] > t1 - 1e-3:
+                continue
+            out[(int(r["i"]), int(r["j"]), round(float(r["tca"]), 3))] = r
+        return out
+
+    h, g = keyset(hyb, 9.0), keyset(grid, 1.0)
+    assert len(g) > 20
+    for k in set(h) ^ set(g):
+        i, j, t = k
+        _, v = orc.propagate(popgen.subset(pop, [i, j]), [t], velocity=True)
+        vrel = np.linalg.norm(v[0, 0] - v[0, 1])
+        assert vrel > 15.6 * 0.999, (k, vrel)       # outside Eq. 1's speed assumption
+    assert len(set(h) ^ set(g)) <= max(2, len(g) // 50)
