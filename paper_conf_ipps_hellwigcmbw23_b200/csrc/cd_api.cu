@@ -493,6 +493,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     int64_t Rsteps = o.round_steps ? (int64_t)o.round_steps
                                    : std::max<int64_t>(1, (int64_t)(qcap / 2 / (size_t)std::max<int64_t>(1, n / 20)));
     unsigned long long conj_before = 0;
+    unsigned long long hyb_before[4] = {0, 0, 0, 0};
     int64_t k = kb;
     while (k < ke) {
         const int64_t Rk = std::min<int64_t>(Rsteps, ke - k);
@@ -545,7 +546,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             if (mode == CD_HYBRID) {
                 CU(launch_hybrid_filter(O, P, q.p, qcap, w.p, wcap, nwork.p, R.conj.p, ocap, ctrl.p,
                                         st, C.lc));
-                CU(launch_hybrid_brent(O, P, w.p, nwork.p, wcap, R.conj.p, ocap, ctrl.p, st, C.lc));
+                CU(launch_brent(O, P, w.p, nwork.p, wcap, R.conj.p, ocap, ctrl.p, st, C.lc));
             } else {
                 CU(launch_prefilter(O, P, q.p, qcap, w.p, wcap, nwork.p, R.conj.p, ocap, ctrl.p, st,
                                     C.lc));
@@ -595,8 +596,16 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             redo = true;
         }
         if (redo) {
-            CU(cudaMemcpyAsync(&ctrl.p->n_conj, &conj_before, sizeof(unsigned long long),
-                               cudaMemcpyHostToDevice, st));
+            // roll the cumulative counters back to the start of the round
+            Ctrl back = *hctrl;
+            back.n_conj = conj_before;
+            back.n_ap = hyb_before[0];
+            back.n_coplanar = hyb_before[1];
+            back.n_path = hyb_before[2];
+            back.n_time = hyb_before[3];
+            back.n_cand = 0;
+            *hctrl = back;
+            CU(cudaMemcpyAsync(ctrl.p, hctrl, sizeof(Ctrl), cudaMemcpyHostToDevice, st));
             CU(cudaStreamSynchronize(st));
             continue;
         }
@@ -619,6 +628,10 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             R.n_cand += hctrl->n_cand;
         }
         conj_before = hctrl->n_conj;
+        hyb_before[0] = hctrl->n_ap;
+        hyb_before[1] = hctrl->n_coplanar;
+        hyb_before[2] = hctrl->n_path;
+        hyb_before[3] = hctrl->n_time;
         if (auto_cell && k == kb) {   // first round done: re-pick the cell edge from the density
             const double m = choose_cell_factor((double)hctrl->n_cand / ((double)Rk * (double)n));
             L = gc * m;

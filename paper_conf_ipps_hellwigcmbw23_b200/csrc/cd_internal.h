@@ -22,10 +22,10 @@ struct Elements {   // device pointers (external order)
     const double *a, *e, *inc, *raan, *argp, *nu0;
 };
 
-// Refinement work item: a candidate that survived the linear pre-filter.
+// Refinement work item: a candidate (or a hybrid time window) for Brent's search.
 struct Work {
-    uint32_t i, j, step, pad;
-    double tw;   // Brent half-window t_w = 2 g_c / min(|v_i|, |v_j|)
+    uint32_t i, j, step, flags;
+    double lo, hi;   // search interval relative to t_k (inside [t0, t1])
 };
 
 // Optional persisting-L2 window applied to a launch (the per-step grid arena: slots, bitmap,

@@ -8,6 +8,7 @@
 #include <cooperative_groups.h>
 
 #include "cd_internal.h"
+#include "cd_refine.cuh"
 
 namespace cg = cooperative_groups;
 using namespace cdk;
@@ -37,19 +38,6 @@ static cudaError_t launch_ex(void (*kern)(KArgs...), dim3 grid, dim3 block, cuda
     cfg.attrs = at;
     cfg.numAttrs = 1;
     return cudaLaunchKernelEx(&cfg, kern, args...);
-}
-
-// Warp-aggregated append: one atomicAdd per group of converged lanes.  The counter keeps
-// counting past `cap` so the host can detect overflow and size the retry.
-template <typename T>
-__device__ __forceinline__ void append(T* buf, size_t cap, unsigned long long* cnt, const T& v)
-{
-    cg::coalesced_group g = cg::coalesced_threads();
-    unsigned long long base = 0;
-    if (g.thread_rank() == 0) base = atomicAdd(cnt, (unsigned long long)g.size());
-    base = g.shfl(base, 0);
-    const unsigned long long idx = base + g.thread_rank();
-    if (idx < cap) buf[idx] = v;
 }
 
 __device__ __forceinline__ void append_count(unsigned long long* cnt)
@@ -407,50 +395,8 @@ __global__ void __launch_bounds__(256) k_prefilter(Orbits O, RefineParams P, con
     unsigned long long nc = ctrl->n_cand;
     if (nc > qcap) nc = qcap;
     const size_t stride = (size_t)gridDim.x * blockDim.x;
-    for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < nc; idx += stride) {
-        const Cand cd = q[idx];
-        const double tk = fma((double)cd.step, P.dt, P.t0);
-        double ri[3], vi[3], rj[3], vj[3];
-        state<true>(O, cd.i, tk, ri, vi);
-        state<true>(O, cd.j, tk, rj, vj);
-        const double dr[3] = {ri[0] - rj[0], ri[1] - rj[1], ri[2] - rj[2]};
-        const double dv[3] = {vi[0] - vj[0], vi[1] - vj[1], vi[2] - vj[2]};
-        const double dv2 = dv[0] * dv[0] + dv[1] * dv[1] + dv[2] * dv[2];
-        const double dr2 = dr[0] * dr[0] + dr[1] * dr[1] + dr[2] * dr[2];
-        if (sqrt(dv2) < 1e-9) {
-            if (sqrt(dr2) < P.d) {
-                Conj cj;
-                cj.i = cd.i; cj.j = cd.j; cj.step = cd.step; cj.flags = 2u;  // CD_FLAG_DEGENERATE
-                cj.tca = tk; cj.pca = sqrt(dr2);
-                append(out, ocap, &ctrl->n_conj, cj);
-            }
-            continue;
-        }
-        const double h = 0.5 * P.dt;
-        double tau = -(dr[0] * dv[0] + dr[1] * dv[1] + dr[2] * dv[2]) / dv2;
-        tau = fmin(fmax(tau, -h), h);
-        const double lx = fma(tau, dv[0], dr[0]), ly = fma(tau, dv[1], dr[1]), lz = fma(tau, dv[2], dr[2]);
-        const double dl = sqrt(lx * lx + ly * ly + lz * lz);
-        const double qi = O.at(kQper, cd.i), qj = O.at(kQper, cd.j);
-        const double amax = kMu / (qi * qi) + kMu / (qj * qj);
-        const double margin = 0.625 * amax * h * h + 1e-6;
-        if (dl - margin >= P.d) continue;
-        const double vi2 = vi[0] * vi[0] + vi[1] * vi[1] + vi[2] * vi[2];
-        const double vj2 = vj[0] * vj[0] + vj[1] * vj[1] + vj[2] * vj[2];
-        Work it;
-        it.i = cd.i; it.j = cd.j; it.step = cd.step; it.pad = 0;
-        it.tw = 2.0 * P.gc / sqrt(fmin(vi2, vj2));
-        append(w, wcap, n_work, it);
-    }
-}
-
-__device__ __forceinline__ double dist2_at(const Orbits& O, uint32_t i, uint32_t j, double t)
-{
-    double a[3], b[3], v[3];
-    state<false>(O, i, t, a, v);
-    state<false>(O, j, t, b, v);
-    const double dx = a[0] - b[0], dy = a[1] - b[1], dz = a[2] - b[2];
-    return fma(dx, dx, fma(dy, dy, dz * dz));
+    for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < nc; idx += stride)
+        grid_refine_item(O, P, q[idx], 0u, w, wcap, n_work, out, ocap, ctrl);
 }
 
 __global__ void __launch_bounds__(128) k_brent(Orbits O, RefineParams P, const Work* __restrict__ w,
@@ -463,8 +409,7 @@ __global__ void __launch_bounds__(128) k_brent(Orbits O, RefineParams P, const W
     for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < nw; idx += stride) {
         const Work it = w[idx];
         const double tk = fma((double)it.step, P.dt, P.t0);
-        double a = fmax(-it.tw, P.t0 - tk);
-        double b = fmin(it.tw, P.t1 - tk);
+        double a = it.lo, b = it.hi;   // relative to t_k, already inside [t0, t1]
         if (!(b > a)) continue;
         const double lo = a, hi = b;
         // Brent's localmin (golden section + successive parabolic interpolation)
@@ -524,7 +469,7 @@ __global__ void __launch_bounds__(128) k_brent(Orbits O, RefineParams P, const W
         const double pca = sqrt(fx);
         if (!(pca < P.d)) continue;
         Conj cj;
-        cj.i = it.i; cj.j = it.j; cj.step = it.step; cj.flags = 0u;
+        cj.i = it.i; cj.j = it.j; cj.step = it.step; cj.flags = it.flags;
         cj.tca = tca; cj.pca = pca;
         append(out, ocap, &ctrl->n_conj, cj);
     }
