@@ -462,6 +462,39 @@ __global__ void __launch_bounds__(128) k_brent(Orbits O, RefineParams P, const W
         // interval-edge rule
         const double tol = eps * fabs(x) + tabs;
         if (x - lo <= 3.0 * tol || hi - x <= 3.0 * tol) continue;
+        // polish: the minimum is the - -> + sign change of g = dr.dv = (1/2) dD^2/dtau.  Brent
+        // locates a flat minimum (slow relative motion) only to ~sqrt(eps) of D^2; bracket the
+        // root of g around x (expanding) and solve it by Illinois regula falsi to 1e-10 s
+        {
+            double hstep = fmax(4.0 * tol, 1e-6), d2a, d2b;
+            double ta = fmax(x - hstep, lo), tb = fmin(x + hstep, hi);
+            double ga = g_at(O, it.i, it.j, tk + ta, d2a), gb = g_at(O, it.i, it.j, tk + tb, d2b);
+            for (int ex = 0; ex < 12 && !(ga < 0.0 && gb >= 0.0); ++ex) {
+                hstep *= 4.0;
+                if (!(ga < 0.0)) { ta = fmax(x - hstep, lo); ga = g_at(O, it.i, it.j, tk + ta, d2a); }
+                if (!(gb >= 0.0)) { tb = fmin(x + hstep, hi); gb = g_at(O, it.i, it.j, tk + tb, d2b); }
+            }
+            if (ga < 0.0 && gb >= 0.0) {
+                int side = 0;
+                for (int k2 = 0; k2 < 80 && tb - ta > 1e-10; ++k2) {
+                    double tc = tb - gb * (tb - ta) / (gb - ga);
+                    if (!(tc > ta && tc < tb)) tc = 0.5 * (ta + tb);
+                    double d2c;
+                    const double gc = g_at(O, it.i, it.j, tk + tc, d2c);
+                    if (gc < 0.0) {
+                        ta = tc; ga = gc;
+                        if (side == -1) gb *= 0.5;
+                        side = -1;
+                    } else {
+                        tb = tc; gb = gc;
+                        if (side == 1) ga *= 0.5;
+                        side = 1;
+                    }
+                }
+                x = 0.5 * (ta + tb);
+                fx = dist2_at(O, it.i, it.j, tk + x);
+            }
+        }
         const double tca = tk + x;
         if (tca < P.t0 || tca > P.t1) continue;
         const double kstar = floor((tca - P.t0) / P.dt + 0.5);
