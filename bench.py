@@ -271,6 +271,52 @@ def run_ours(args):
         units = float(u.item())
     value = units / (tot_ms / 1e3)
 
+    # the hybrid variant (coarse grid at dt_h + filter chain) over the same window, same slicing
+    hyb = None
+    if args.variant == "grid" and not args.no_hybrid and cfg.dt_hybrid:
+        Kh = int(np.floor((cfg.t1 - cfg.t0) / cfg.dt_hybrid)) + 1
+        hms, hst = [], []
+        for s in range(args.warmup + args.steps):
+            q = (s * world + rank) % S
+            E = cds._Elements(dpop)
+            st = cds.cd_stats()
+            opt = cds.make_options(rank=q, n_ranks=S, device=dev.index, stream=stream.cuda_stream,
+                                   inputs_on_device=True, outputs_on_device=True)
+            import ctypes as C
+            opt.stats = C.pointer(st)
+            out = cds.cd_conjunctions()
+            flush.zero_()
+            torch.cuda.synchronize()
+            barrier()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            cds._check(cds.cd_screen_ex(E.s, E.n, cfg.t0, cfg.t1, cfg.dt_hybrid, cfg.d, cds.CD_HYBRID,
+                                        opt, out))
+            recs = cdist.device_records_to_tensor(out, dev)
+            if world > 1:
+                recs = cdist.merge_conjunctions(recs, stream=stream.cuda_stream)
+            cds.cd_conjunctions_free(out)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            if s >= args.warmup:
+                hms.append(e0.elapsed_time(e1))
+                hst.append(st.as_dict())
+        htot = float(np.sum(hms))
+        if world > 1:
+            t = torch.tensor([htot], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            htot = float(t.item())
+        hunits = float(n) * sum(h["steps"] for h in hst) * world
+        hyb = {"variant": "hybrid", "dt_s": cfg.dt_hybrid, "steps_in_window": Kh,
+               "value": hunits / (htot / 1e3), "unit": "object-steps/s (coarse steps)",
+               "wall_s_window": htot / 1e3,
+               "coarse_candidates": int(sum(h["candidates"] for h in hst)),
+               "conjunctions": int(sum(h["conjunctions"] for h in hst)),
+               "filter": {k: int(sum(h[k] for h in hst)) for k in
+                          ("hybrid_ap_rejected", "hybrid_coplanar", "hybrid_path_rejected",
+                           "hybrid_time_rejected", "refined")}}
+
     # end to end through the public API with HOST buffers (pinned inputs, results to host)
     e2e_ms = []
     pin = {k: torch.from_numpy(v).pin_memory() for k, v in pop.items()}
@@ -351,7 +397,7 @@ def run_ours(args):
             "step_ms": {"min": float(np.min(times)), "median": float(np.median(times)),
                         "max": float(np.max(times))},
             "clocks": clk.summary(), "e2e": e2e, "gpu_launches": launches,
-            "roofline": roof, "cpu_baseline": cpu}
+            "roofline": roof, "cpu_baseline": cpu, "hybrid": hyb}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
@@ -381,6 +427,7 @@ def main():
     ap.add_argument("--n", type=int, default=None, help="override object count (testing)")
     ap.add_argument("--no-profile", dest="profile", action="store_false")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-hybrid", action="store_true")
     ap.add_argument("--cpu-steps", type=int, default=128)
     ap.add_argument("--ref-steps", type=int, default=None)
     ap.add_argument("--e2e-steps", type=int, default=None)
