@@ -131,6 +131,10 @@ typedef struct {
     int profile_phases;       /* N > 0: time every N-th launch of each phase into cd_stats     */
     int l2_persist;           /* pin the per-step grid tables in a persisting-L2 window (default
                                  0; raises cudaLimitPersistingL2CacheSize for the device)      */
+    int grid_table;           /* per-step grid structure: 1 = the paper's open-addressing hash
+                                 map (64-bit keys, linear probing, CAS, per-cell lists);
+                                 2 = chained spatial hash (lists per hashed bucket, one atomic
+                                 exchange per object); 0 = default (2).  Results are identical. */
     cd_stats* stats;          /* optional output                                              */
 } cd_options;
 

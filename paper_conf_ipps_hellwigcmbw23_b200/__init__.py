@@ -81,7 +81,7 @@ class cd_options(C.Structure):
                 ("inputs_on_device", C.c_int), ("outputs_on_device", C.c_int),
                 ("kepler_points", C.c_int), ("cell_factor", C.c_double),
                 ("batch_object_steps", C.c_size_t), ("round_steps", C.c_size_t),
-                ("profile_phases", C.c_int), ("l2_persist", C.c_int),
+                ("profile_phases", C.c_int), ("l2_persist", C.c_int), ("grid_table", C.c_int),
                 ("stats", C.POINTER(cd_stats))]
 
 
@@ -207,7 +207,7 @@ class _Elements:
 def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None, stream=None,
                  cell_factor=None, batch_object_steps=None, round_steps=None,
                  outputs_on_device=False, inputs_on_device=False, profile_phases=False,
-                 l2_persist=None):
+                 l2_persist=None, grid_table=None):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -231,6 +231,8 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
     o.profile_phases = int(profile_phases)
     if l2_persist is not None:
         o.l2_persist = int(bool(l2_persist))
+    if grid_table is not None:
+        o.grid_table = int(grid_table)
     return o
 
 

@@ -409,6 +409,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     g.gc2 = gc * gc;
     g.reach = gc * (1.0 + 1e-9) + 1e-9;
     g.halfshell = L < 2.0 * gc ? 1 : 0;
+    g.max_walk = (uint32_t)std::min<int64_t>(n + 1, 0xfffffffe);
     RefineParams P{t0, t1, dt, d, gc};
 
     R.conj.st = R.cand.st = st;
@@ -424,9 +425,16 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     // two entry buffers.  Launch i of a round builds batch b+1 (slot set (b+1) % 2 with tag
     // (b+1) % 126 + 1, bitmap set (b+1) % 3, entries (b+1) % 2), scans batch b and zeroes bitmap set
     // (b+2) % 3.  Slot sets are zeroed only when their tags wrap.
-    const uint64_t nbits = std::max<uint64_t>(next_pow2((uint64_t)n * 32), 1024);   // >= 32 bits/object
-    const uint32_t bwords = (uint32_t)(nbits / 32);
-    const size_t slot_bytes = sizeof(Slot) * (size_t)Bmax * M;
+    // grid structure: 1 = the paper's open-addressing map (slots + occupancy bitmap);
+    // 2 = chained spatial hash (bucket heads only; default, measured faster)
+    const bool chained = o.grid_table != 1;
+#ifndef CD_CHAIN_FACTOR
+#define CD_CHAIN_FACTOR 4
+#endif
+    const uint64_t nbits = chained ? std::max<uint64_t>(next_pow2((uint64_t)n * CD_CHAIN_FACTOR), 1024) * 32
+                                   : std::max<uint64_t>(next_pow2((uint64_t)n * 32), 1024);
+    const uint32_t bwords = (uint32_t)(nbits / 32);   // chained: one 32-bit head per word
+    const size_t slot_bytes = chained ? 0 : sizeof(Slot) * (size_t)Bmax * M;
     const size_t bit_bytes = ((sizeof(uint32_t) * (size_t)Bmax * bwords + 255) / 256) * 256;
     const size_t ent_bytes = sizeof(Entry) * (size_t)Bmax * n;
     const size_t tab_bytes = 2 * slot_bytes + 3 * bit_bytes;
@@ -440,7 +448,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     Entry* entbuf[2] = {reinterpret_cast<Entry*>(arena.p + tab_bytes),
                         reinterpret_cast<Entry*>(arena.p + tab_bytes + ent_bytes)};
     auto tab_of = [&](uint64_t b) {
-        return GridTab{slotset[b % 2], bitset[b % 3], (uint32_t)(nbits - 1), bwords};
+        return GridTab{slotset[b % 2], bitset[b % 3], chained ? bwords - 1u : (uint32_t)(nbits - 1), bwords};
     };
     auto tag_of = [](uint64_t b) { return (uint32_t)(b % kMaxTag) + 1u; };
     uint64_t batch_no = 0;
@@ -514,7 +522,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                 sa.ctrl = ctrl.p;
                 const uint64_t bb = batch_no + (uint64_t)i;   // batch built in this launch
                 if (i < J) {
-                    if (bb % kMaxTag < 2 && bb >= 2) {
+                    if (!chained && bb % kMaxTag < 2 && bb >= 2) {
                         // this slot set's tags wrap with this batch: zero it (its last scan, of
                         // batch bb - 2, finished in the previous launch)
                         CU(cudaMemsetAsync(slotset[bb % 2], 0, slot_bytes, st));
@@ -535,6 +543,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                 sa.zero_bits = bitset[(bb + 1) % 3];   // batch bb - 2's bitmaps, next built by bb + 1
                 sa.zero_bits_words = bwords;
                 sa.zero_depth = Bmax;
+                sa.chained = chained ? 1 : 0;
                 C.pt.start(i < J && i == 0 ? kPhPropagate : kPhScan);
                 CU(launch_step(sa, &win, st, C.lc));
                 C.pt.stop();
@@ -733,6 +742,7 @@ void cd_options_init(cd_options* o)
     o->n_ranks = 1;
     o->cell_factor = 0.0;   // auto (1.0 = the paper's cell edge g_c, 27-cell neighbourhood)
     o->l2_persist = 0;
+    o->grid_table = 0;
 }
 
 cd_status cd_screen(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,

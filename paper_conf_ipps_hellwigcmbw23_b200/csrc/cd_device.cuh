@@ -315,9 +315,10 @@ constexpr int kTagShift = 57;
 constexpr uint32_t kMaxTag = 126;
 constexpr uint32_t kNil = 0xffffffffu;
 
-__device__ __forceinline__ uint64_t pack_key(int64_t cx, int64_t cy, int64_t cz)
+__device__ __forceinline__ uint64_t pack_key(int cx, int cy, int cz)
 {
-    return uint64_t(cx + kKeyBias) | (uint64_t(cy + kKeyBias) << 19) | (uint64_t(cz + kKeyBias) << 38);
+    return uint64_t(uint32_t(cx + (int)kKeyBias)) | (uint64_t(uint32_t(cy + (int)kKeyBias)) << 19) |
+           (uint64_t(uint32_t(cz + (int)kKeyBias)) << 38);
 }
 
 // MurmurHash3 64-bit finaliser (footnote 3: smhasher)
@@ -338,15 +339,39 @@ struct GridGeom {
     double reach;        // g_c (1 + 1e-9) + 1e-9: ball radius used to pick the probed cells
     int halfshell;       // 1: own cell + 13 half-shell neighbours (L < 2 g_c); 0: the cells
                          // overlapping the ball |x - p| < g_c (L >= 2 g_c)
+    uint32_t max_walk;   // list-walk bound (n): guards against a corrupted list
 };
 
-__device__ __forceinline__ bool cell_of(const GridGeom& g, const double p[3], int64_t c[3])
+// Cell of position p: c = floor((p - o) / L) per axis (R7); frac = (p - o)/L - c in [0, 1).
+// Returns false outside the key range.
+__device__ __forceinline__ bool cell_of(const GridGeom& g, const double p[3], int c[3], double* frac = nullptr)
 {
-    c[0] = (int64_t)floor((p[0] - g.ox) * g.inv_cell);
-    c[1] = (int64_t)floor((p[1] - g.oy) * g.inv_cell);
-    c[2] = (int64_t)floor((p[2] - g.oz) * g.inv_cell);
-    return c[0] >= -kCellMax && c[0] <= kCellMax && c[1] >= -kCellMax && c[1] <= kCellMax &&
-           c[2] >= -kCellMax && c[2] <= kCellMax;
+    const double u[3] = {(p[0] - g.ox) * g.inv_cell, (p[1] - g.oy) * g.inv_cell, (p[2] - g.oz) * g.inv_cell};
+    bool ok = true;
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+        const double f = floor(u[a]);
+        ok = ok && f >= -(double)kCellMax && f <= (double)kCellMax;
+        c[a] = ok ? (int)f : 0;
+        if (frac) frac[a] = u[a] - f;
+    }
+    return ok;
+}
+
+// Occupancy-bitmap hash of a cell from per-axis products (so the scan can combine neighbour
+// cells with two XORs): h = mix(cx*A ^ cy*B ^ cz*C).  Any fixed hash is valid for the bitmap;
+// only its uniformity matters (false-positive rate).
+constexpr uint32_t kHX = 0x9E3779B1u, kHY = 0x85EBCA77u, kHZ = 0xC2B2AE3Du;
+__device__ __forceinline__ uint32_t bit_mix(uint32_t h)
+{
+    h ^= h >> 15;
+    h *= 0x2C1B3C6Du;
+    h ^= h >> 12;
+    return h;
+}
+__device__ __forceinline__ uint32_t bit_hash(int cx, int cy, int cz)
+{
+    return bit_mix((uint32_t)cx * kHX ^ (uint32_t)cy * kHY ^ (uint32_t)cz * kHZ);
 }
 
 // Grid entry (Fig. 6: id, coordinates, next); the id is the entry index.
@@ -410,23 +435,9 @@ __device__ __forceinline__ uint32_t grid_insert(Slot* slots, uint64_t mask, unsi
     }
 }
 
-// Per-step occupancy bitmap over hashed cell keys: 32 bits per object, so a probe of an empty
-// cell (the common case) is one 4-byte load from a 4 MB (at 1M objects) L2-resident array;
-// false positives (~3 %) only cost a table probe.  MurmurHash3 fmix32 of the folded key.
-__device__ __forceinline__ uint32_t fmix32(uint32_t h)
-{
-    h ^= h >> 16;
-    h *= 0x85ebca6bu;
-    h ^= h >> 13;
-    h *= 0xc2b2ae35u;
-    h ^= h >> 16;
-    return h;
-}
-__device__ __forceinline__ uint32_t bit_of(unsigned long long key)
-{
-    return fmix32((uint32_t)key + 0x9e3779b9u * (uint32_t)(key >> 32));
-}
-
+// Per-step occupancy bitmap: 32 bits per object, set at insertion with bit_hash(cell); a probe
+// of an empty cell (the common case) is one 4-byte load from a small L2-resident array; false
+// positives (~3 %) only cost a table probe.
 struct GridTab {
     Slot* slots;      // M slots per step
     uint32_t* bits;   // bwords words per step

@@ -177,21 +177,41 @@ cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long l
 // (Eq. 2) and its occupancy bitmap; the entry {x, y, z, next} (Fig. 6) is
 // written once, coalesced.  kClass0: objects [0, n0) (e <= 0.01: lean N = 4 Contour path).
 // ---------------------------------------------------------------------------------------
-template <bool kClass0>
+template <bool kClass0, bool kChained>
 __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, const GridTab& tab,
                                          Entry* __restrict__ ents, uint64_t mask, int64_t k0, int s,
                                          int64_t r, double t0, double dt, uint32_t tag, Ctrl* ctrl)
 {
     const double t = fma((double)(k0 + s), dt, t0);
     double p[3], v[3];
+#ifdef CD_ABL_NO_PROP   // ablation (timing experiments only): position from one record column
+    p[0] = O.at(kAPx, r) + t; p[1] = O.at(kAPy, r); p[2] = O.at(kAPz, r);
+#else
     state<false, kClass0 ? 0 : -1>(O, r, t, p, v);
-    int64_t c[3];
+#endif
+    int c[3];
     uint32_t next = kNil;
-    if (cell_of(g, p, c)) {
+    if (kChained && cell_of(g, p, c)) {
+        // chained spatial hash: push onto the list of bucket hash(cell) -- one atomic exchange;
+        // heads hold index + 1 (0 = empty bucket)
+        const uint32_t b = bit_hash(c[0], c[1], c[2]) & tab.bmask;
+#ifndef CD_ABL_NO_EXCH
+        const uint32_t prev = atomicExch(tab.bits + (size_t)s * tab.bwords + b, (uint32_t)r + 1u);
+        next = prev ? prev - 1u : kNil;
+#else
+        next = b == 0xffffffffu ? 0u : kNil;
+#endif
+    } else if (!kChained && cell_of(g, p, c)) {
         const unsigned long long key = pack_key(c[0], c[1], c[2]);
-        const uint32_t hb = bit_of(key) & tab.bmask;
+        const uint32_t hb = bit_hash(c[0], c[1], c[2]) & tab.bmask;
+#ifndef CD_ABL_NO_RED
         atomicOr(tab.bits + (size_t)s * tab.bwords + (hb >> 5), 1u << (hb & 31));
+#endif
+#ifndef CD_ABL_NO_CAS
         next = grid_insert(tab.slots + (size_t)s * (mask + 1), mask, key, tag, (uint32_t)r);
+#else
+        next = (uint32_t)(key & 0) | kNil;
+#endif
     } else {
         ctrl->err_range = 1;
     }
@@ -201,7 +221,20 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
     en.z = p[2];
     en.next = next;
     en.pad = 0;
+#ifdef CD_STREAM_ENTRIES
+    // written once here, read once (coalesced) by the next launch's scan: stream past L2 so the
+    // randomly accessed slot table and bitmaps keep it
+    double4* dst = reinterpret_cast<double4*>(ents + (size_t)s * O.n + r);
+    double4 v4;
+    v4.x = en.x;
+    v4.y = en.y;
+    v4.z = en.z;
+    v4.w = __longlong_as_double((long long)en.next);
+    __stcs(reinterpret_cast<double2*>(dst), make_double2(v4.x, v4.y));
+    __stcs(reinterpret_cast<double2*>(dst) + 1, make_double2(v4.z, v4.w));
+#else
     ents[(size_t)s * O.n + r] = en;
+#endif
 }
 
 // ---------------------------------------------------------------------------------------
@@ -240,36 +273,27 @@ __device__ __forceinline__ void walk(const GridGeom& g, const Entry* __restrict_
                                      uint32_t r, const double p[3], bool only_greater, uint32_t step,
                                      Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
 {
+    uint32_t guard = g.max_walk;   // a list is never longer than n; a cycle would be a bug
     while (j != kNil) {
+        if (guard-- == 0) {
+            ctrl->err_internal = 1;
+            return;
+        }
         const Entry ej = E[j];
         if (!only_greater || j > r) test_pair(g, r, j, p, ej, step, q, qcap, ctrl);
         j = ej.next;
     }
 }
 
-// Probe NP cells: issue every bitmap load first (independent 4-byte loads), then probe the
-// table only for set bits and walk the hits.
-template <int NP, typename KeyFn>
-__device__ __forceinline__ void probe_group(const GridGeom& g, const Slot* __restrict__ slots,
-                                            const uint32_t* __restrict__ bits, uint32_t bmask,
-                                            uint64_t mask, uint32_t tag, uint32_t valid, KeyFn keyf,
-                                            const Entry* __restrict__ E, uint32_t r, const double p[3],
-                                            bool only_greater, uint32_t step, Cand* __restrict__ q,
-                                            size_t qcap, Ctrl* ctrl)
+// Scan one object against the cells listed by (dx, dy, dz) offsets of its own cell: every bitmap
+// load is issued before any is resolved; set bits probe the table and walk the cell's list.
+__device__ __forceinline__ void probe_cell(const GridGeom& g, const Slot* __restrict__ slots,
+                                           uint64_t mask, uint32_t tag, int cx, int cy, int cz,
+                                           const Entry* __restrict__ E, uint32_t r, const double p[3],
+                                           bool only_greater, uint32_t step, Cand* __restrict__ q,
+                                           size_t qcap, Ctrl* ctrl)
 {
-    uint32_t hit = 0;
-#pragma unroll
-    for (int i = 0; i < NP; ++i) {
-        if ((valid >> i) & 1u) {
-            const uint32_t hb = bit_of(keyf(i)) & bmask;
-            hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << i;
-        }
-    }
-    while (hit) {
-        const int i = __ffs(hit) - 1;
-        hit &= hit - 1;
-        walk(g, E, grid_find(slots, mask, keyf(i), tag), r, p, only_greater, step, q, qcap, ctrl);
-    }
+    walk(g, E, grid_find(slots, mask, pack_key(cx, cy, cz), tag), r, p, only_greater, step, q, qcap, ctrl);
 }
 
 __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
@@ -279,40 +303,161 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
 {
     const Slot* slots = tab.slots + (size_t)s * (mask + 1);
     const uint32_t* bits = tab.bits + (size_t)s * tab.bwords;
+    const uint32_t bmask = tab.bmask;
+    const Entry* E = ents + (size_t)s * n;
+    const uint32_t step = (uint32_t)(k0 + s);
+#ifdef CD_STREAM_ENTRIES
+    Entry me;
+    {
+        const double2 a = __ldcs(reinterpret_cast<const double2*>(E + r));
+        const double2 b = __ldcs(reinterpret_cast<const double2*>(E + r) + 1);
+        me.x = a.x;
+        me.y = a.y;
+        me.z = b.x;
+        me.next = (uint32_t)__double_as_longlong(b.y);
+        me.pad = 0;
+    }
+#else
+    const Entry me = E[r];
+#endif
+    const double p[3] = {me.x, me.y, me.z};
+    int c[3];
+    double fr[3];
+    if (!cell_of(g, p, c, fr)) return;
+    // (1) own cell: successors in the object's own list
+    walk(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
+    // (2) other cells
+    const uint32_t hx0 = (uint32_t)c[0] * kHX, hy0 = (uint32_t)c[1] * kHY, hz0 = (uint32_t)c[2] * kHZ;
+    if (g.halfshell) {
+        uint32_t hit = 0;
+#pragma unroll
+        for (int o = 1; o < 14; ++o) {
+            const uint32_t hb = bit_mix((hx0 + (uint32_t)kHalfShell[o][0] * kHX) ^
+                                        (hy0 + (uint32_t)kHalfShell[o][1] * kHY) ^
+                                        (hz0 + (uint32_t)kHalfShell[o][2] * kHZ)) & bmask;
+            hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << o;
+        }
+        while (hit) {
+            const int o = __ffs(hit) - 1;
+            hit &= hit - 1;
+            probe_cell(g, slots, mask, tag, c[0] + kHalfShell[o][0], c[1] + kHalfShell[o][1],
+                       c[2] + kHalfShell[o][2], E, (uint32_t)r, p, false, step, q, qcap, ctrl);
+        }
+    } else {
+        // ball mode: per axis the other overlapped cell (c - 1 if the ball crosses the lower
+        // face, c + 1 if the upper); frac * L is the distance to the lower face
+        const double rl = g.reach * g.inv_cell;
+        const int d0 = fr[0] < rl ? -1 : (fr[0] > 1.0 - rl ? 1 : 0);
+        const int d1 = fr[1] < rl ? -1 : (fr[1] > 1.0 - rl ? 1 : 0);
+        const int d2 = fr[2] < rl ? -1 : (fr[2] > 1.0 - rl ? 1 : 0);
+        // (c +- 1 stays inside the 19-bit key range because |c| <= kCellMax = 2^18 - 2)
+        const uint32_t hx1 = hx0 + (uint32_t)d0 * kHX, hy1 = hy0 + (uint32_t)d1 * kHY,
+                       hz1 = hz0 + (uint32_t)d2 * kHZ;
+        // cell c + (b0 d0, b1 d1, b2 d2), b = 1..7, exists iff every axis set in b has d != 0
+        const uint32_t valid = (d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu) & 0xFEu;
+        uint32_t hit = 0;
+#pragma unroll
+        for (int b = 1; b < 8; ++b) {
+            const uint32_t hb = bit_mix(((b & 1) ? hx1 : hx0) ^ ((b & 2) ? hy1 : hy0) ^
+                                        ((b & 4) ? hz1 : hz0)) & bmask;
+            if ((valid >> b) & 1u) hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << b;
+        }
+        while (hit) {
+            const int b = __ffs(hit) - 1;
+            hit &= hit - 1;
+            probe_cell(g, slots, mask, tag, c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0),
+                       c[2] + ((b & 4) ? d2 : 0), E, (uint32_t)r, p, true, step, q, qcap, ctrl);
+        }
+    }
+}
+
+// Chained spatial hash (alternative grid structure): the lists hang off bucket hash(cell), so a
+// bucket may also hold objects of other cells -- the exact distance test filters them.
+//  * pairs inside the object's own bucket (same cell, or a colliding cell) are found by the
+//    later-inserted object walking its own list successors (no probe);
+//  * every other bucket of its neighbourhood (own cell's 0-7 ball cells, or all 27 cells when
+//    L < 2 g_c), distinct and different from the own bucket, is walked in full and a pair is
+//    reported only from its smaller id -- for a pair closer than g_c in different buckets each
+//    object's neighbourhood contains the other's cell, so the smaller id sees it exactly once.
+__device__ __forceinline__ void walk_bucket(const GridGeom& g, const Entry* __restrict__ E,
+                                            uint32_t h, uint32_t r, uint32_t my_next, const double p[3],
+                                            uint32_t step, Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
+{
+    uint32_t j = h ? h - 1u : kNil;
+    uint32_t guard = g.max_walk;
+    while (j != kNil) {
+        if (guard-- == 0) {
+            ctrl->err_internal = 1;
+            return;
+        }
+        if (j == r) {
+            j = my_next;
+            continue;
+        }
+        const Entry ej = E[j];
+        if (j > r) test_pair(g, r, j, p, ej, step, q, qcap, ctrl);
+        j = ej.next;
+    }
+}
+
+__device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab& tab,
+                                                const Entry* __restrict__ ents, int64_t n, int64_t k0,
+                                                int s, int64_t r, Cand* __restrict__ q, size_t qcap,
+                                                Ctrl* ctrl)
+{
+    const uint32_t* heads = tab.bits + (size_t)s * tab.bwords;
+    const uint32_t hmask = tab.bmask;
     const Entry* E = ents + (size_t)s * n;
     const uint32_t step = (uint32_t)(k0 + s);
     const Entry me = E[r];
     const double p[3] = {me.x, me.y, me.z};
-    int64_t c[3];
-    if (!cell_of(g, p, c)) return;
-    // (1) own cell: successors in the object's own list
+    int c[3];
+    double fr[3];
+    if (!cell_of(g, p, c, fr)) return;
+    // own bucket: successors only, every pair once (by the later-inserted object)
     walk(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
-    // (2) other cells
-    if (g.halfshell) {
-        auto k1 = [=](int i) { return pack_key(c[0] + kHalfShell[1 + i][0], c[1] + kHalfShell[1 + i][1],
-                                               c[2] + kHalfShell[1 + i][2]); };
-        auto k2 = [=](int i) { return pack_key(c[0] + kHalfShell[8 + i][0], c[1] + kHalfShell[8 + i][1],
-                                               c[2] + kHalfShell[8 + i][2]); };
-        probe_group<7>(g, slots, bits, tab.bmask, mask, tag, 0x7Fu, k1, E, (uint32_t)r, p, false, step, q, qcap, ctrl);
-        probe_group<6>(g, slots, bits, tab.bmask, mask, tag, 0x3Fu, k2, E, (uint32_t)r, p, false, step, q, qcap, ctrl);
-    } else {
-        int64_t lo[3], hi[3];
-        const double pl[3] = {p[0] - g.reach, p[1] - g.reach, p[2] - g.reach};
-        const double ph[3] = {p[0] + g.reach, p[1] + g.reach, p[2] + g.reach};
-        if (!cell_of(g, pl, lo) || !cell_of(g, ph, hi)) return;
-        // per axis: the other overlapped cell (c - 1 or c + 1), or none
-        const int64_t d0 = lo[0] < c[0] ? -1 : (hi[0] > c[0] ? 1 : 0);
-        const int64_t d1 = lo[1] < c[1] ? -1 : (hi[1] > c[1] ? 1 : 0);
-        const int64_t d2 = lo[2] < c[2] ? -1 : (hi[2] > c[2] ? 1 : 0);
-        // cell c + (b0 d0, b1 d1, b2 d2), b = 1..7 (bit i <-> b = i + 1), exists iff every axis set
-        // in b has d != 0
-        const uint32_t valid = (((d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu)) >> 1) & 0x7Fu;
-        auto kb = [=](int i) {
-            const int b = i + 1;
-            return pack_key(c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0), c[2] + ((b & 4) ? d2 : 0));
-        };
-        probe_group<7>(g, slots, bits, tab.bmask, mask, tag, valid, kb, E, (uint32_t)r, p, true, step, q, qcap, ctrl);
+    const uint32_t hx0 = (uint32_t)c[0] * kHX, hy0 = (uint32_t)c[1] * kHY, hz0 = (uint32_t)c[2] * kHZ;
+    const uint32_t own = bit_mix(hx0 ^ hy0 ^ hz0) & hmask;
+    if (g.halfshell) {   // L < 2 g_c: all 26 neighbour cells (rare configuration; local arrays)
+        uint32_t bk[26];
+        int nb = 0;
+        for (int dx = -1; dx <= 1; ++dx)
+            for (int dy = -1; dy <= 1; ++dy)
+                for (int dz = -1; dz <= 1; ++dz) {
+                    const uint32_t b = bit_mix((hx0 + (uint32_t)dx * kHX) ^ (hy0 + (uint32_t)dy * kHY) ^
+                                               (hz0 + (uint32_t)dz * kHZ)) & hmask;
+                    bool dup = b == own;
+                    for (int k = 0; k < nb; ++k) dup = dup || bk[k] == b;
+                    if (!dup) bk[nb++] = b;
+                }
+        for (int k = 0; k < nb; ++k)
+            walk_bucket(g, E, __ldg(heads + bk[k]), (uint32_t)r, me.next, p, step, q, qcap, ctrl);
+        return;
     }
+    const double rl = g.reach * g.inv_cell;
+    const int d0 = fr[0] < rl ? -1 : (fr[0] > 1.0 - rl ? 1 : 0);
+    const int d1 = fr[1] < rl ? -1 : (fr[1] > 1.0 - rl ? 1 : 0);
+    const int d2 = fr[2] < rl ? -1 : (fr[2] > 1.0 - rl ? 1 : 0);
+    uint32_t valid = (d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu) & 0xFEu;
+    if (!valid) return;
+    const uint32_t hx1 = hx0 + (uint32_t)d0 * kHX, hy1 = hy0 + (uint32_t)d1 * kHY,
+                   hz1 = hz0 + (uint32_t)d2 * kHZ;
+    uint32_t bk[8];
+    bk[0] = own;
+#pragma unroll
+    for (int b = 1; b < 8; ++b)
+        bk[b] = bit_mix(((b & 1) ? hx1 : hx0) ^ ((b & 2) ? hy1 : hy0) ^ ((b & 4) ? hz1 : hz0)) & hmask;
+#pragma unroll
+    for (int b = 1; b < 8; ++b)   // distinct buckets, other than the own bucket
+#pragma unroll
+        for (int k = 0; k < b; ++k)
+            if ((k == 0 || ((valid >> k) & 1u)) && bk[b] == bk[k]) valid &= ~(1u << b);
+    uint32_t hd[8];
+#pragma unroll
+    for (int b = 1; b < 8; ++b) hd[b] = ((valid >> b) & 1u) ? __ldg(heads + bk[b]) : 0u;
+#pragma unroll
+    for (int b = 1; b < 8; ++b)
+        if (hd[b]) walk_bucket(g, E, hd[b], (uint32_t)r, me.next, p, step, q, qcap, ctrl);
 }
 
 // ---------------------------------------------------------------------------------------
@@ -326,23 +471,27 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
 #ifndef CD_STEP_MINB
 #define CD_STEP_MINB 6
 #endif
+template <bool kChained>
 __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
 {
     const int64_t bx = blockIdx.x;
     const int64_t nA = a.build_B * a.nbA, nB = a.build_B * a.nbB;
+#ifdef CD_ABL_NO_BUILD
+    if (bx < nA + nB) return;
+#endif
     if (bx < nA) {
         const int s = (int)(bx / a.nbA);
         const int64_t r = (bx % a.nbA) * 256 + threadIdx.x;
         if (r < a.O.n0)
-            do_build<true>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0, a.dt,
-                           a.build_tag, a.ctrl);
+            do_build<true, kChained>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
+                                     a.dt, a.build_tag, a.ctrl);
     } else if (bx < nA + nB) {
         const int64_t b2 = bx - nA;
         const int s = (int)(b2 / a.nbB);
         const int64_t r = a.O.n0 + (b2 % a.nbB) * 256 + threadIdx.x;
         if (r < a.O.n)
-            do_build<false>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0, a.dt,
-                            a.build_tag, a.ctrl);
+            do_build<false, kChained>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
+                                      a.dt, a.build_tag, a.ctrl);
     } else {
         const int64_t b3 = bx - nA - nB;
         // zero the bitmap set of batch b + 2 (all Bmax tables), grid-stride over role-C threads
@@ -352,11 +501,18 @@ __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
         uint4* zb = reinterpret_cast<uint4*>(a.zero_bits);
         for (int64_t i = tid; i < nw4; i += nth) zb[i] = make_uint4(0u, 0u, 0u, 0u);
         if (a.scan_B == 0) return;
+#ifdef CD_ABL_NO_SCAN
+        return;
+#endif
         const int s = (int)(b3 / a.nbC);
         const int64_t r = (b3 % a.nbC) * 256 + threadIdx.x;
-        if (r < a.O.n)
-            do_scan(a.g, a.scan_tab, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r, a.scan_tag, a.q,
-                    a.qcap, a.ctrl);
+        if (r < a.O.n) {
+            if (kChained)
+                do_scan_chained(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.q, a.qcap, a.ctrl);
+            else
+                do_scan(a.g, a.scan_tab, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r, a.scan_tag, a.q,
+                        a.qcap, a.ctrl);
+        }
     }
 }
 
@@ -370,7 +526,8 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
     const int64_t blocks = a.build_B * (a.nbA + a.nbB) + a.nCblocks;
     if (blocks == 0) return cudaSuccess;
     lc.bump();
-    return launch_ex(k_step, dim3((unsigned)blocks), dim3(256), st, win, a);
+    if (a.chained) return launch_ex(k_step<true>, dim3((unsigned)blocks), dim3(256), st, win, a);
+    return launch_ex(k_step<false>, dim3((unsigned)blocks), dim3(256), st, win, a);
 }
 
 // ---------------------------------------------------------------------------------------

@@ -96,6 +96,8 @@ def test_candidates_ragged_sizes(n, steps, d):
 
 
 @pytest.mark.parametrize("kw", [dict(grid_origin=(1234.5, -987.25, 55.125)), dict(cell_factor=1.0),
+                                dict(grid_table=1), dict(grid_table=1, cell_factor=1.0),
+                                dict(grid_table=2, cell_factor=1.0), dict(grid_table=1, round_steps=5),
                                 dict(cell_factor=2.0), dict(cell_factor=1.5, grid_origin=(-3e3, 7.5, 1e4)),
                                 dict(cell_factor=3.7), dict(batch_object_steps=1),
                                 dict(round_steps=7), dict(batch_object_steps=10 ** 7)])
@@ -180,7 +182,8 @@ def test_screen_ragged_parity(n, steps, d):
     assert res["matched"] > 0
 
 
-def test_screen_dense_shell_many_conjunctions():
+@pytest.mark.parametrize("table", [1, 2])
+def test_screen_dense_shell_many_conjunctions(table):
     """A compact shell with many encounters per step (exercises queue growth and refinement)."""
     rng = np.random.default_rng(3)
     n = 6000
@@ -189,7 +192,7 @@ def test_screen_dense_shell_many_conjunctions():
            "argp": rng.uniform(0, 2 * math.pi, n), "nu0": rng.uniform(0, 2 * math.pi, n)}
     d, t1 = 5.0, 200.0
     gc = oracle.cell_size(d, 1.0)
-    Cg = cds.screen(pop, 0.0, t1, 1.0, d, round_steps=13)
+    Cg = cds.screen(pop, 0.0, t1, 1.0, d, round_steps=13, grid_table=table)
     Ko = oracle.candidates_grid(pop, 0.0, t1, 1.0, gc)
     Co = oracle.conjunctions(pop, 0.0, t1, 1.0, d, gc, Ko)
     res = parity.compare_conjunctions(pop, Cg, Co, 0.0, t1, 1.0, d, gc)

@@ -15,7 +15,8 @@ def main():
     ap.add_argument("--variant", default="grid")
     ap.add_argument("--cell", default="1,2,3,4,5,6,8")
     ap.add_argument("--batch", default="0")
-    ap.add_argument("--persist", default="1")
+    ap.add_argument("--persist", default="0")
+    ap.add_argument("--table", default="0")
     args = ap.parse_args()
     import torch
     import paper_conf_ipps_hellwigcmbw23_b200 as cds
@@ -27,9 +28,10 @@ def main():
     t1 = t0 + (args.steps - 1) * dt
     ref = None
     for pers in [int(x) for x in args.persist.split(",")]:
+     for tbl in [int(x) for x in args.table.split(",")]:
       for b in [int(x) for x in args.batch.split(",")]:
         for cf in [float(x) for x in args.cell.split(",")]:
-            kw = dict(cell_factor=cf, profile_phases=True, l2_persist=pers)
+            kw = dict(cell_factor=cf, profile_phases=True, l2_persist=pers, grid_table=tbl)
             if b:
                 kw["batch_object_steps"] = b
             cds.screen(dpop, t0, t0 + 20 * dt, dt, cfg.d, mode=args.variant, **kw)  # warm
@@ -38,7 +40,7 @@ def main():
                 ref = res
             same = bool(len(res) == len(ref) and (res[["i", "j", "step"]] == ref[["i", "j", "step"]]).all())
             k = st["steps"]
-            out = {"cell": cf, "batch": b, "persist": pers, "ms_per_step_total": st["ms_total"] / k,
+            out = {"cell": cf, "table": tbl, "batch": b, "persist": pers, "ms_per_step_total": st["ms_total"] / k,
                    "us_clear": 1e3 * st["ms_clear"] / k, "us_prop": 1e3 * st["ms_propagate"] / k,
                    "us_insert": 1e3 * st["ms_insert"] / k, "us_scan": 1e3 * st["ms_scan"] / k,
                    "us_refine": 1e3 * st["ms_refine"] / k, "cand": st["candidates"],
