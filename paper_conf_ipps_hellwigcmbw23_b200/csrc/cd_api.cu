@@ -11,6 +11,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -30,6 +31,20 @@ using namespace cdh;
 namespace {
 
 thread_local std::string g_err;
+
+// host-side timeline for diagnosis (CD_DEBUG_TIMING=1)
+struct DebugClock {
+    bool on = getenv("CD_DEBUG_TIMING") != nullptr;
+    std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now();
+    void mark(const char* what, long long a = -1, long long b = -1) const
+    {
+        if (!on) return;
+        const double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        fprintf(stderr, "[cd %9.3f ms] %s %lld %lld\n", ms, what, a, b);
+    }
+};
+thread_local DebugClock* g_dbg = nullptr;
+#define DBG(...) do { if (g_dbg) g_dbg->mark(__VA_ARGS__); } while (0)
 
 cd_status fail(cd_status s, const char* fmt, ...)
 {
@@ -410,7 +425,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     g.reach = gc * (1.0 + 1e-9) + 1e-9;
     g.halfshell = L < 2.0 * gc ? 1 : 0;
     g.max_walk = (uint32_t)std::min<int64_t>(n + 1, 0xfffffffe);
-    RefineParams P{t0, t1, dt, d, gc};
+    RefineParams P{t0, t1, dt, d, gc, nullptr};
 
     R.conj.st = R.cand.st = st;
     if (ke <= kb || n < 2) return CD_OK;
@@ -425,21 +440,30 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     // two entry buffers.  Launch i of a round builds batch b+1 (slot set (b+1) % 2 with tag
     // (b+1) % 126 + 1, bitmap set (b+1) % 3, entries (b+1) % 2), scans batch b and zeroes bitmap set
     // (b+2) % 3.  Slot sets are zeroed only when their tags wrap.
-    // grid structure: 1 = the paper's open-addressing map (slots + occupancy bitmap);
-    // 2 = chained spatial hash (bucket heads only; default, measured faster)
-    const bool chained = o.grid_table != 1;
+    // grid structure: 1 = the paper's open-addressing map (slots + occupancy bitmap); 2 = chained
+    // spatial hash (bucket heads only); 0 = per geometry: chained in ball mode (L >= 2 g_c, where
+    // it is measured faster), open addressing in half-shell mode (L < 2 g_c, where chaining would
+    // walk all 26 neighbour buckets from both sides).  Both are allocated under 0, so the mode
+    // can follow the cell edge chosen after the first round.
+    const bool can_chain = o.grid_table != 1, can_open = o.grid_table != 2;
 #ifndef CD_CHAIN_FACTOR
 #define CD_CHAIN_FACTOR 4
 #endif
-    const uint64_t nbits = chained ? std::max<uint64_t>(next_pow2((uint64_t)n * CD_CHAIN_FACTOR), 1024) * 32
-                                   : std::max<uint64_t>(next_pow2((uint64_t)n * 32), 1024);
-    const uint32_t bwords = (uint32_t)(nbits / 32);   // chained: one 32-bit head per word
-    const size_t slot_bytes = chained ? 0 : sizeof(Slot) * (size_t)Bmax * M;
+    const uint64_t chain_words = can_chain ? std::max<uint64_t>(next_pow2((uint64_t)n * CD_CHAIN_FACTOR), 1024) : 0;
+    const uint64_t nbits = std::max<uint64_t>(next_pow2((uint64_t)n * 32), 1024);   // open: >= 32 bits/object
+    const uint32_t bwords = (uint32_t)std::max<uint64_t>(chain_words, can_open ? nbits / 32 : 0);
+    const size_t slot_bytes = can_open ? sizeof(Slot) * (size_t)Bmax * M : 0;
+    auto pick_chained = [&](const GridGeom& gg) {
+        return o.grid_table == 2 || (o.grid_table == 0 && !gg.halfshell);
+    };
+    bool chained = pick_chained(g);
     const size_t bit_bytes = ((sizeof(uint32_t) * (size_t)Bmax * bwords + 255) / 256) * 256;
     const size_t ent_bytes = sizeof(Entry) * (size_t)Bmax * n;
     const size_t tab_bytes = 2 * slot_bytes + 3 * bit_bytes;
     DBuf<unsigned char> arena(st);
+    DBG("run: alloc arena", (long long)(tab_bytes + 2 * ent_bytes));
     CU(arena.alloc(tab_bytes + 2 * ent_bytes));
+    DBG("run: arena allocated");
     CU(cudaMemsetAsync(arena.p, 0, tab_bytes, st));
     Slot* slotset[2] = {reinterpret_cast<Slot*>(arena.p), reinterpret_cast<Slot*>(arena.p + slot_bytes)};
     uint32_t* bitset[3];
@@ -448,7 +472,8 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     Entry* entbuf[2] = {reinterpret_cast<Entry*>(arena.p + tab_bytes),
                         reinterpret_cast<Entry*>(arena.p + tab_bytes + ent_bytes)};
     auto tab_of = [&](uint64_t b) {
-        return GridTab{slotset[b % 2], bitset[b % 3], chained ? bwords - 1u : (uint32_t)(nbits - 1), bwords};
+        return GridTab{slotset[b % 2], bitset[b % 3],
+                       chained ? (uint32_t)(chain_words - 1) : (uint32_t)(nbits - 1), bwords};
     };
     auto tag_of = [](uint64_t b) { return (uint32_t)(b % kMaxTag) + 1u; };
     uint64_t batch_no = 0;
@@ -485,13 +510,21 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     size_t ccap = want == Want::Cand ? (size_t(1) << 20) : 0;
     if (want == Want::Cand) CU(R.cand.alloc(ccap));
 
+    DBuf<unsigned char> hrec(st);
+    if (mode == CD_HYBRID && want == Want::Conj) {
+        CU(hrec.alloc(hybrid_record_bytes() * (size_t)n));
+        CU(launch_build_hybrid_records(O, hrec.p, st, C.lc));
+        P.hrec = hrec.p;
+    }
     DBuf<Ctrl> ctrl(st);
     CU(ctrl.alloc(1));
     CU(cudaMemsetAsync(ctrl.p, 0, sizeof(Ctrl), st));
     DBuf<unsigned long long> nwork(st);
     CU(nwork.alloc(1));
     Ctrl* hctrl = nullptr;
+    DBG("run: queues allocated");
     CU(cudaMallocHost((void**)&hctrl, sizeof(Ctrl) + sizeof(unsigned long long)));
+    DBG("run: pinned ctrl");
     struct HostFree {
         void* p;
         ~HostFree() { cudaFreeHost(p); }
@@ -522,7 +555,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                 sa.ctrl = ctrl.p;
                 const uint64_t bb = batch_no + (uint64_t)i;   // batch built in this launch
                 if (i < J) {
-                    if (!chained && bb % kMaxTag < 2 && bb >= 2) {
+                    if (can_open && bb % kMaxTag < 2 && bb >= 2) {
                         // this slot set's tags wrap with this batch: zero it (its last scan, of
                         // batch bb - 2, finished in the previous launch)
                         CU(cudaMemsetAsync(slotset[bb % 2], 0, slot_bytes, st));
@@ -565,7 +598,9 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         }
         CU(cudaMemcpyAsync(hctrl, ctrl.p, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
         CU(cudaMemcpyAsync(hnwork, nwork.p, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+        DBG("round: enqueued", (long long)k, (long long)Rk);
         CU(cudaStreamSynchronize(st));
+        DBG("round: synced", (long long)k, (long long)Rk);
         C.pt.harvest();
         if (hctrl->err_internal)
             return fail(CD_EINTERNAL, "internal: a grid cell list did not terminate");
@@ -647,9 +682,17 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             if (L < gc * (1.0 + 1e-12)) L = gc * (1.0 + 1e-12);
             g.inv_cell = 1.0 / L;
             g.halfshell = L < 2.0 * gc ? 1 : 0;
+            chained = pick_chained(g);
         }
         if (!o.round_steps) {
             const double rate = std::max(1.0, (double)hctrl->n_cand / (double)Rk);
+            // dense candidate rates (hybrid): grow the queue so a round spans >= 64 steps (each
+            // round ends with a host sync), within a 2^28-entry (3 GB) cap
+            const double wanted = rate * 64.0 * 1.25;
+            if (wanted > (double)qcap && qcap < (size_t(1) << 28)) {
+                qcap = (size_t)std::min(wanted, (double)(size_t(1) << 28));
+                CU(q.alloc(qcap));   // (the work-item buffer grows on demand via the retry path)
+            }
             Rsteps = std::max<int64_t>(1, std::min<int64_t>(1 << 16, (int64_t)(0.5 * qcap / rate)));
         }
         k += Rk;
@@ -682,15 +725,21 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
     TRY(validate_scalars(n, t0, t1, dt, d, o, &K));
     cd_stats stats;
     memset(&stats, 0, sizeof stats);
+    DebugClock dbg;
+    g_dbg = &dbg;
+    struct Reset { ~Reset() { g_dbg = nullptr; } } reset_dbg;
     Call C;
     TRY(C.begin(o));
+    DBG("screen: begin");
     Result R;
     DBuf<Conj> sorted(C.st);
     {
         OrbitSet S;
         if (n > 0) TRY(prepare_orbits(C, el, n, o, S));
         else if (!el) return fail(CD_EINVAL, "elements must be non-NULL");
+        DBG("screen: orbits ready");
         TRY(run(C, S, t0, t1, dt, d, mode, o, K, Want::Conj, R, stats));
+        DBG("screen: run done");
         if (R.n_conj) {
             C.pt.start(kPhFinalize);
             CU(sorted.alloc(R.n_conj));
@@ -712,8 +761,10 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
             own->p = h;
         }
     }
+    DBG("screen: finalized");
     CU(cudaEventRecord(C.ev1, C.st));
     CU(cudaEventSynchronize(C.ev1));
+    DBG("screen: end synced");
     float ms = 0.f;
     cudaEventElapsedTime(&ms, C.ev0, C.ev1);
     stats.ms_total = ms;

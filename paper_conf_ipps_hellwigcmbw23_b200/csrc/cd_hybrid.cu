@@ -27,10 +27,12 @@ namespace {
 constexpr double kPiH = 3.14159265358979323846;
 constexpr double kTwoPiH = 6.28318530717958647692;
 
-struct HOrbit {
+struct __align__(128) HOrbit {   // one 128-byte line per object (compact gather in the filter)
     double e, q, Q, p, nm, M0;
     double P[3], Qv[3], h[3];
+    double pad;
 };
+static_assert(sizeof(HOrbit) == 128, "HOrbit must be one 128-byte line");
 
 __device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o)
 {
@@ -51,6 +53,7 @@ __device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o)
     o.p = a * (1.0 - o.e) * (1.0 + o.e);
     o.nm = O.at(kNm, r);
     o.M0 = O.at(kM0, r);
+    o.pad = 0.0;
 }
 
 __device__ __forceinline__ double mean_of_true(double f, double e)
@@ -112,19 +115,27 @@ __device__ __forceinline__ void count1(unsigned long long* cnt)
 
 }  // namespace
 
+__global__ void k_build_hrec(Orbits O, HOrbit* __restrict__ hr)
+{
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (r >= O.n) return;
+    HOrbit o;
+    horbit(O, r, o);
+    hr[r] = o;
+}
+
 __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P, const Cand* __restrict__ q,
                                                        size_t qcap, Work* __restrict__ w, size_t wcap,
                                                        unsigned long long* n_work,
                                                        Conj* __restrict__ out, size_t ocap, Ctrl* ctrl)
 {
+    const HOrbit* __restrict__ hr = static_cast<const HOrbit*>(P.hrec);
     unsigned long long nc = ctrl->n_cand;
     if (nc > qcap) nc = qcap;
     const size_t stride = (size_t)gridDim.x * blockDim.x;
     for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < nc; idx += stride) {
         const Cand cd = q[idx];
-        HOrbit A, B;
-        horbit(O, cd.i, A);
-        horbit(O, cd.j, B);
+        const HOrbit A = hr[cd.i], B = hr[cd.j];
         const double d = P.d;
         // apogee / perigee
         if (fmax(A.q, B.q) - fmin(A.Q, B.Q) > d) {
@@ -188,6 +199,15 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
         if (!any_node) count1(&ctrl->n_path);
         else if (nwin == 0) count1(&ctrl->n_time);
     }
+}
+
+size_t hybrid_record_bytes() { return sizeof(HOrbit); }
+
+cudaError_t launch_build_hybrid_records(const Orbits& O, void* hrec, cudaStream_t st, LaunchCount& lc)
+{
+    k_build_hrec<<<(unsigned)((O.n + 127) / 128), 128, 0, st>>>(O, static_cast<HOrbit*>(hrec));
+    lc.bump();
+    return cudaGetLastError();
 }
 
 cudaError_t launch_hybrid_filter(const Orbits& O, const RefineParams& p, const Cand* q, size_t qcap,

@@ -37,6 +37,7 @@ struct L2Win {
 
 struct RefineParams {
     double t0, t1, dt, d, gc;
+    const void* hrec = nullptr;   // hybrid: compact per-object filter records
 };
 
 // ---- precompute (a1) -------------------------------------------------------------------
