@@ -454,6 +454,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     const uint32_t bwords = (uint32_t)std::max<uint64_t>(chain_words, can_open ? nbits / 32 : 0);
     const size_t slot_bytes = can_open ? sizeof(Slot) * (size_t)Bmax * M : 0;
     auto pick_chained = [&](const GridGeom& gg) {
+        if (n > (int64_t)kMaxChainN) return false;   // 24-bit head indices
         return o.grid_table == 2 || (o.grid_table == 0 && !gg.halfshell);
     };
     bool chained = pick_chained(g);
@@ -475,7 +476,10 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         return GridTab{slotset[b % 2], bitset[b % 3],
                        chained ? (uint32_t)(chain_words - 1) : (uint32_t)(nbits - 1), bwords};
     };
-    auto tag_of = [](uint64_t b) { return (uint32_t)(b % kMaxTag) + 1u; };
+    // key tags (open map, 7 bits) / head epochs (chained grid, 8 bits): never 0 (= cleared)
+    auto tag_of = [&](uint64_t b) {
+        return chained ? (uint32_t)(b % 255u) + 1u : (uint32_t)(b % kMaxTag) + 1u;
+    };
     uint64_t batch_no = 0;
     // persisting-L2 window over the slot and bitmap sets (they take the random atomics and
     // probes; records, entries and candidate writes stream past them)
@@ -555,6 +559,12 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                 sa.ctrl = ctrl.p;
                 const uint64_t bb = batch_no + (uint64_t)i;   // batch built in this launch
                 if (i < J) {
+                    if (chained && bb % 255u < 3 && bb >= 3) {
+                        // head set bb % 3 is used by batches of one residue mod 3; its epochs
+                        // (bb % 255 + 1) would repeat within the next 255 batches: zero it (its
+                        // last scan, of batch bb - 3, finished two launches ago)
+                        CU(cudaMemsetAsync(bitset[bb % 3], 0, bit_bytes, st));
+                    }
                     if (can_open && bb % kMaxTag < 2 && bb >= 2) {
                         // this slot set's tags wrap with this batch: zero it (its last scan, of
                         // batch bb - 2, finished in the previous launch)
@@ -575,7 +585,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                 }
                 sa.zero_bits = bitset[(bb + 1) % 3];   // batch bb - 2's bitmaps, next built by bb + 1
                 sa.zero_bits_words = bwords;
-                sa.zero_depth = Bmax;
+                sa.zero_depth = chained ? 0 : Bmax;   // chained heads are epoch-tagged
                 sa.chained = chained ? 1 : 0;
                 C.pt.start(i < J && i == 0 ? kPhPropagate : kPhScan);
                 CU(launch_step(sa, &win, st, C.lc));

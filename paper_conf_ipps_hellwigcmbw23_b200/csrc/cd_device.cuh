@@ -374,6 +374,21 @@ __device__ __forceinline__ uint32_t bit_hash(int cx, int cy, int cz)
     return bit_mix((uint32_t)cx * kHX ^ (uint32_t)cy * kHY ^ (uint32_t)cz * kHZ);
 }
 
+// Chained-grid bucket of a cell: hash of its aligned 2x2x2 block (floor(c/2) per axis) in the
+// high bits, the cell's parity (c mod 2 per axis) in the low 3 bits.  The <= 8 cells a ball of
+// radius g_c <= L/2 overlaps have pairwise different parities, so their buckets are always
+// distinct (no de-duplication), and the 8 cells of a block share one 32-byte sector of heads.
+__device__ __forceinline__ uint32_t chain_bucket(int cx, int cy, int cz, uint32_t hmask)
+{
+    const uint32_t blk = bit_mix((uint32_t)(cx >> 1) * kHX ^ (uint32_t)(cy >> 1) * kHY ^
+                                 (uint32_t)(cz >> 1) * kHZ);
+    return ((blk << 3) | (uint32_t)(cx & 1) | ((uint32_t)(cy & 1) << 1) | ((uint32_t)(cz & 1) << 2)) & hmask;
+}
+// Chained-grid heads: (epoch << 24) | (index + 1); a head of another epoch is an empty bucket,
+// so the head arrays are never cleared per step (zeroed only when the 8-bit epoch wraps).
+constexpr uint32_t kEpochShift = 24, kIdxMask = (1u << 24) - 1u;
+constexpr uint32_t kMaxChainN = (1u << 24) - 2u;   // chained grid needs n < 2^24 - 1
+
 // Grid entry (Fig. 6: id, coordinates, next); the id is the entry index.
 struct __align__(32) Entry {
     double x, y, z;

@@ -194,10 +194,11 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
     if (kChained && cell_of(g, p, c)) {
         // chained spatial hash: push onto the list of bucket hash(cell) -- one atomic exchange;
         // heads hold index + 1 (0 = empty bucket)
-        const uint32_t b = bit_hash(c[0], c[1], c[2]) & tab.bmask;
+        const uint32_t b = chain_bucket(c[0], c[1], c[2], tab.bmask);
 #ifndef CD_ABL_NO_EXCH
-        const uint32_t prev = atomicExch(tab.bits + (size_t)s * tab.bwords + b, (uint32_t)r + 1u);
-        next = prev ? prev - 1u : kNil;
+        const uint32_t prev = atomicExch(tab.bits + (size_t)s * tab.bwords + b,
+                                         (tag << kEpochShift) | ((uint32_t)r + 1u));
+        next = ((prev >> kEpochShift) == tag && (prev & kIdxMask)) ? (prev & kIdxMask) - 1u : kNil;
 #else
         next = b == 0xffffffffu ? 0u : kNil;
 #endif
@@ -380,10 +381,11 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
 //    reported only from its smaller id -- for a pair closer than g_c in different buckets each
 //    object's neighbourhood contains the other's cell, so the smaller id sees it exactly once.
 __device__ __forceinline__ void walk_bucket(const GridGeom& g, const Entry* __restrict__ E,
-                                            uint32_t h, uint32_t r, uint32_t my_next, const double p[3],
-                                            uint32_t step, Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
+                                            uint32_t h, uint32_t epoch, uint32_t r, uint32_t my_next,
+                                            const double p[3], uint32_t step, Cand* __restrict__ q,
+                                            size_t qcap, Ctrl* ctrl)
 {
-    uint32_t j = h ? h - 1u : kNil;
+    uint32_t j = ((h >> kEpochShift) == epoch && (h & kIdxMask)) ? (h & kIdxMask) - 1u : kNil;
     uint32_t guard = g.max_walk;
     while (j != kNil) {
         if (guard-- == 0) {
@@ -402,8 +404,8 @@ __device__ __forceinline__ void walk_bucket(const GridGeom& g, const Entry* __re
 
 __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab& tab,
                                                 const Entry* __restrict__ ents, int64_t n, int64_t k0,
-                                                int s, int64_t r, Cand* __restrict__ q, size_t qcap,
-                                                Ctrl* ctrl)
+                                                int s, int64_t r, uint32_t epoch, Cand* __restrict__ q,
+                                                size_t qcap, Ctrl* ctrl)
 {
     const uint32_t* heads = tab.bits + (size_t)s * tab.bwords;
     const uint32_t hmask = tab.bmask;
@@ -416,48 +418,39 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
     if (!cell_of(g, p, c, fr)) return;
     // own bucket: successors only, every pair once (by the later-inserted object)
     walk(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
-    const uint32_t hx0 = (uint32_t)c[0] * kHX, hy0 = (uint32_t)c[1] * kHY, hz0 = (uint32_t)c[2] * kHZ;
-    const uint32_t own = bit_mix(hx0 ^ hy0 ^ hz0) & hmask;
     if (g.halfshell) {   // L < 2 g_c: all 26 neighbour cells (rare configuration; local arrays)
+        const uint32_t own = chain_bucket(c[0], c[1], c[2], hmask);
         uint32_t bk[26];
         int nb = 0;
         for (int dx = -1; dx <= 1; ++dx)
             for (int dy = -1; dy <= 1; ++dy)
                 for (int dz = -1; dz <= 1; ++dz) {
-                    const uint32_t b = bit_mix((hx0 + (uint32_t)dx * kHX) ^ (hy0 + (uint32_t)dy * kHY) ^
-                                               (hz0 + (uint32_t)dz * kHZ)) & hmask;
+                    const uint32_t b = chain_bucket(c[0] + dx, c[1] + dy, c[2] + dz, hmask);
                     bool dup = b == own;
                     for (int k = 0; k < nb; ++k) dup = dup || bk[k] == b;
                     if (!dup) bk[nb++] = b;
                 }
         for (int k = 0; k < nb; ++k)
-            walk_bucket(g, E, __ldg(heads + bk[k]), (uint32_t)r, me.next, p, step, q, qcap, ctrl);
+            walk_bucket(g, E, __ldg(heads + bk[k]), epoch, (uint32_t)r, me.next, p, step, q, qcap, ctrl);
         return;
     }
     const double rl = g.reach * g.inv_cell;
     const int d0 = fr[0] < rl ? -1 : (fr[0] > 1.0 - rl ? 1 : 0);
     const int d1 = fr[1] < rl ? -1 : (fr[1] > 1.0 - rl ? 1 : 0);
     const int d2 = fr[2] < rl ? -1 : (fr[2] > 1.0 - rl ? 1 : 0);
-    uint32_t valid = (d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu) & 0xFEu;
+    const uint32_t valid = (d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu) & 0xFEu;
     if (!valid) return;
-    const uint32_t hx1 = hx0 + (uint32_t)d0 * kHX, hy1 = hy0 + (uint32_t)d1 * kHY,
-                   hz1 = hz0 + (uint32_t)d2 * kHZ;
-    uint32_t bk[8];
-    bk[0] = own;
-#pragma unroll
-    for (int b = 1; b < 8; ++b)
-        bk[b] = bit_mix(((b & 1) ? hx1 : hx0) ^ ((b & 2) ? hy1 : hy0) ^ ((b & 4) ? hz1 : hz0)) & hmask;
-#pragma unroll
-    for (int b = 1; b < 8; ++b)   // distinct buckets, other than the own bucket
-#pragma unroll
-        for (int k = 0; k < b; ++k)
-            if ((k == 0 || ((valid >> k) & 1u)) && bk[b] == bk[k]) valid &= ~(1u << b);
+    // the ball's cells differ pairwise in parity -> distinct buckets, no de-duplication
     uint32_t hd[8];
 #pragma unroll
-    for (int b = 1; b < 8; ++b) hd[b] = ((valid >> b) & 1u) ? __ldg(heads + bk[b]) : 0u;
+    for (int b = 1; b < 8; ++b)
+        hd[b] = ((valid >> b) & 1u)
+                    ? __ldg(heads + chain_bucket(c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0),
+                                                 c[2] + ((b & 4) ? d2 : 0), hmask))
+                    : 0u;
 #pragma unroll
     for (int b = 1; b < 8; ++b)
-        if (hd[b]) walk_bucket(g, E, hd[b], (uint32_t)r, me.next, p, step, q, qcap, ctrl);
+        if (hd[b]) walk_bucket(g, E, hd[b], epoch, (uint32_t)r, me.next, p, step, q, qcap, ctrl);
 }
 
 // ---------------------------------------------------------------------------------------
@@ -474,41 +467,44 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
 template <bool kChained>
 __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
 {
-    const int64_t bx = blockIdx.x;
-    const int64_t nA = a.build_B * a.nbA, nB = a.build_B * a.nbB;
+    const uint32_t bx = blockIdx.x;
+    const uint32_t nbA = (uint32_t)a.nbA, nbB = (uint32_t)a.nbB, nbC = (uint32_t)a.nbC;
+    const uint32_t nA = (uint32_t)a.build_B * nbA, nB = (uint32_t)a.build_B * nbB;
 #ifdef CD_ABL_NO_BUILD
     if (bx < nA + nB) return;
 #endif
     if (bx < nA) {
-        const int s = (int)(bx / a.nbA);
-        const int64_t r = (bx % a.nbA) * 256 + threadIdx.x;
+        const int s = (int)(bx / nbA);
+        const int64_t r = (int64_t)(bx % nbA) * 256 + threadIdx.x;
         if (r < a.O.n0)
             do_build<true, kChained>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
                                      a.dt, a.build_tag, a.ctrl);
     } else if (bx < nA + nB) {
-        const int64_t b2 = bx - nA;
-        const int s = (int)(b2 / a.nbB);
-        const int64_t r = a.O.n0 + (b2 % a.nbB) * 256 + threadIdx.x;
+        const uint32_t b2 = bx - nA;
+        const int s = (int)(b2 / nbB);
+        const int64_t r = a.O.n0 + (int64_t)(b2 % nbB) * 256 + threadIdx.x;
         if (r < a.O.n)
             do_build<false, kChained>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
                                       a.dt, a.build_tag, a.ctrl);
     } else {
-        const int64_t b3 = bx - nA - nB;
+        const uint32_t b3 = bx - nA - nB;
         // zero the bitmap set of batch b + 2 (all Bmax tables), grid-stride over role-C threads
-        const int64_t tid = b3 * 256 + threadIdx.x;
+        const int64_t tid = (int64_t)b3 * 256 + threadIdx.x;
         const int64_t nth = a.nCblocks * 256;
         const int64_t nw4 = (int64_t)a.zero_depth * a.zero_bits_words / 4;
         uint4* zb = reinterpret_cast<uint4*>(a.zero_bits);
-        for (int64_t i = tid; i < nw4; i += nth) zb[i] = make_uint4(0u, 0u, 0u, 0u);
+        if (!kChained)   // chained heads are epoch-tagged: nothing to clear
+            for (int64_t i = tid; i < nw4; i += nth) zb[i] = make_uint4(0u, 0u, 0u, 0u);
         if (a.scan_B == 0) return;
 #ifdef CD_ABL_NO_SCAN
         return;
 #endif
-        const int s = (int)(b3 / a.nbC);
-        const int64_t r = (b3 % a.nbC) * 256 + threadIdx.x;
+        const int s = (int)(b3 / nbC);
+        const int64_t r = (int64_t)(b3 % nbC) * 256 + threadIdx.x;
         if (r < a.O.n) {
             if (kChained)
-                do_scan_chained(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.q, a.qcap, a.ctrl);
+                do_scan_chained(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
+                                a.qcap, a.ctrl);
             else
                 do_scan(a.g, a.scan_tab, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r, a.scan_tag, a.q,
                         a.qcap, a.ctrl);
