@@ -359,7 +359,8 @@ def run_ours(args):
         # k_step (fused build + scan) runs as the "propagate" phase (first, build-only launch of
         # each round) and the "scan" phase (all other launches); its algorithmic bytes are
         # SURVEY 8(d)'s 296 B per object-step (insert 48 + detect 248)
-        # sampled: every PROFILE_EVERY-th launch of a phase is timed (events on the call's stream)
+        # the step loop of every round is one event span (the launches overlap under
+        # programmatic dependent launch): average launch = span time / launches in the spans
         ms_smp = sum(s_["ms_scan"] + s_["ms_propagate"] for s_ in stats)
         nl_smp = sum(s_["launches_scan"] + s_["launches_propagate"] for s_ in stats)
         nl = sum(s_["step_launches"] for s_ in stats)

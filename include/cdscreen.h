@@ -106,7 +106,9 @@ typedef struct {
     double ms_total;           /* device time of the call (CUDA events on the call's stream)  */
     /* per-phase device time and timed-launch counts, filled only when cd_options.profile_phases
        > 0 (CUDA events on the call's stream around every profile_phases-th launch of a phase;
-       no extra syncs): average launch duration = ms_X / launches_X                            */
+       no extra syncs): average launch duration = ms_X / launches_X.  The fused step kernel is
+       timed as one span per round (ms_scan / launches_scan = its pipelined launch period; its
+       launches overlap under programmatic dependent launch), ms_propagate stays 0            */
     double ms_clear, ms_propagate, ms_insert, ms_scan, ms_refine, ms_finalize, ms_precompute;
     uint64_t launches_clear, launches_propagate, launches_insert, launches_scan, launches_refine;
     uint64_t step_launches;    /* all launches of the fused step kernel (timed or not)         */

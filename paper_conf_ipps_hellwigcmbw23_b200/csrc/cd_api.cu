@@ -132,7 +132,7 @@ struct PhaseTimer {
     cudaStream_t st = nullptr;
     std::vector<cudaEvent_t> pool;
     size_t used = 0;
-    struct Mark { int ph; size_t a, b; };
+    struct Mark { int ph; size_t a, b; uint64_t nl; };
     std::vector<Mark> marks;
     double ms[kNPhase] = {};
     uint64_t launches[kNPhase] = {};
@@ -166,7 +166,25 @@ struct PhaseTimer {
         if (!on || cur < 0) return;
         const size_t b = used;
         cudaEventRecord(ev(), st);
-        marks.push_back({cur, cur_a, b});
+        marks.push_back({cur, cur_a, b, 1});
+        cur = -1;
+    }
+    // unsampled span over nl back-to-back launches of one phase (a round's step loop): the
+    // launches keep overlapping each other (programmatic dependent launch) inside the span
+    void span_start(int ph)
+    {
+        if (!on) return;
+        cur = ph;
+        cur_a = used;
+        cudaEventRecord(ev(), st);
+    }
+    void span_stop(uint64_t nl)
+    {
+        if (!on || cur < 0) return;
+        const size_t b = used;
+        cudaEventRecord(ev(), st);
+        marks.push_back({cur, cur_a, b, nl});
+        calls[cur] += nl;
         cur = -1;
     }
     // call after the stream has been synchronised
@@ -176,7 +194,7 @@ struct PhaseTimer {
         for (const Mark& m : marks) {
             float x = 0.f;
             if (cudaEventElapsedTime(&x, pool[m.a], pool[m.b]) == cudaSuccess) ms[m.ph] += x;
-            launches[m.ph] += 1;
+            launches[m.ph] += m.nl;
         }
         marks.clear();
         used = 0;
@@ -462,16 +480,19 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     const size_t ent_bytes = sizeof(Entry) * (size_t)Bmax * n;
     const size_t tab_bytes = 2 * slot_bytes + 3 * bit_bytes;
     DBuf<unsigned char> arena(st);
-    DBG("run: alloc arena", (long long)(tab_bytes + 2 * ent_bytes));
-    CU(arena.alloc(tab_bytes + 2 * ent_bytes));
+    DBG("run: alloc arena", (long long)(tab_bytes + 3 * ent_bytes));
+    CU(arena.alloc(tab_bytes + 3 * ent_bytes));
     DBG("run: arena allocated");
     CU(cudaMemsetAsync(arena.p, 0, tab_bytes, st));
     Slot* slotset[2] = {reinterpret_cast<Slot*>(arena.p), reinterpret_cast<Slot*>(arena.p + slot_bytes)};
     uint32_t* bitset[3];
     for (int h = 0; h < 3; ++h)
         bitset[h] = reinterpret_cast<uint32_t*>(arena.p + 2 * slot_bytes + h * bit_bytes);
-    Entry* entbuf[2] = {reinterpret_cast<Entry*>(arena.p + tab_bytes),
-                        reinterpret_cast<Entry*>(arena.p + tab_bytes + ent_bytes)};
+    // three entry buffers: with programmatic dependent launch, launch i + 1 builds batch b + 2
+    // while launch i may still scan batch b (and build b + 1)
+    Entry* entbuf[3];
+    for (int h = 0; h < 3; ++h) entbuf[h] = reinterpret_cast<Entry*>(arena.p + tab_bytes + h * ent_bytes);
+    static const bool no_pdl = getenv("CD_NO_PDL") != nullptr;   // A/B switch for experiments
     auto tab_of = [&](uint64_t b) {
         return GridTab{slotset[b % 2], bitset[b % 3],
                        chained ? (uint32_t)(chain_words - 1) : (uint32_t)(nbits - 1), bwords};
@@ -573,24 +594,25 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                     sa.build_k0 = k + i * Bmax;
                     sa.build_B = std::min<int64_t>(Bmax, k + Rk - sa.build_k0);
                     sa.build_tab = tab_of(bb);
-                    sa.build_ents = entbuf[bb % 2];
+                    sa.build_ents = entbuf[bb % 3];
                     sa.build_tag = tag_of(bb);
                 }
                 if (i > 0) {
                     sa.scan_k0 = k + (i - 1) * Bmax;
                     sa.scan_B = std::min<int64_t>(Bmax, k + Rk - sa.scan_k0);
                     sa.scan_tab = tab_of(bb - 1);
-                    sa.scan_ents = entbuf[(bb - 1) % 2];
+                    sa.scan_ents = entbuf[(bb - 1) % 3];
                     sa.scan_tag = tag_of(bb - 1);
                 }
                 sa.zero_bits = bitset[(bb + 1) % 3];   // batch bb - 2's bitmaps, next built by bb + 1
                 sa.zero_bits_words = bwords;
                 sa.zero_depth = chained ? 0 : Bmax;   // chained heads are epoch-tagged
                 sa.chained = chained ? 1 : 0;
-                C.pt.start(i < J && i == 0 ? kPhPropagate : kPhScan);
+                sa.pdl = chained && !no_pdl ? 1 : 0;
+                if (i == 0) C.pt.span_start(kPhScan);
                 CU(launch_step(sa, &win, st, C.lc));
-                C.pt.stop();
             }
+            C.pt.span_stop((uint64_t)J + 1);
             batch_no += (uint64_t)J;
         }
         if (want == Want::Conj) {

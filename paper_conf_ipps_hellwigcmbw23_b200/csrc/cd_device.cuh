@@ -384,6 +384,13 @@ __device__ __forceinline__ uint32_t chain_bucket(int cx, int cy, int cz, uint32_
                                  (uint32_t)(cz >> 1) * kHZ);
     return ((blk << 3) | (uint32_t)(cx & 1) | ((uint32_t)(cy & 1) << 1) | ((uint32_t)(cz & 1) << 2)) & hmask;
 }
+// Cell tag stored with each chained-grid entry: the cell's coordinates mod 1024 per axis.  Two
+// cells of one 3x3x3 neighbourhood never share a tag, so a walk can tell the probed cell's
+// entries from those of a colliding neighbour cell without recomputing cells from positions.
+__device__ __forceinline__ uint32_t cell_tag(int cx, int cy, int cz)
+{
+    return ((uint32_t)cx & 0x3FFu) | (((uint32_t)cy & 0x3FFu) << 10) | (((uint32_t)cz & 0x3FFu) << 20);
+}
 // Chained-grid heads: (epoch << 24) | (index + 1); a head of another epoch is an empty bucket,
 // so the head arrays are never cleared per step (zeroed only when the 8-bit epoch wraps).
 constexpr uint32_t kEpochShift = 24, kIdxMask = (1u << 24) - 1u;
@@ -393,7 +400,7 @@ constexpr uint32_t kMaxChainN = (1u << 24) - 2u;   // chained grid needs n < 2^2
 struct __align__(32) Entry {
     double x, y, z;
     uint32_t next;
-    uint32_t pad;
+    uint32_t tag;    // chained grid: cell_tag of the entry's cell (open map: unused)
 };
 
 // Hash grid of one step.  Open addressing over M = 2^m >= 2n slots,

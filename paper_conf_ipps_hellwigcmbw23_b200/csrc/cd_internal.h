@@ -77,6 +77,7 @@ struct StepArgs {
     int64_t nbA, nbB, nbC;       // blocks per step of roles A, B, C (filled by launch_step)
     int64_t nCblocks;            // role-C blocks in the launch
     int chained;                 // 1: chained spatial hash (heads in the bitmap arrays)
+    int pdl;                     // 1: programmatic dependent launch (chained grid only)
 };
 cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCount& lc);
 

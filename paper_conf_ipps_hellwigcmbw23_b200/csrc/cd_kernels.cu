@@ -20,11 +20,14 @@ std::atomic<uint64_t> g_launches{0};
 static inline unsigned blocks_for(int64_t n, int t) { return (unsigned)((n + t - 1) / t); }
 
 // Launch with an optional persisting-L2 access-policy window (per-launch attribute).
+// With pdl, the launch may begin while the previous kernel in the stream is still running
+// (programmatic dependent launch); the kernel orders its dependent part with griddepcontrol.wait.
 template <typename... KArgs, typename... Args>
 static cudaError_t launch_ex(void (*kern)(KArgs...), dim3 grid, dim3 block, cudaStream_t st,
-                             const L2Win* win, Args... args)
+                             const L2Win* win, bool pdl, Args... args)
 {
-    if (!win || !win->on) {
+    const bool w = win && win->on;
+    if (!w && !pdl) {
         kern<<<grid, block, 0, st>>>(args...);
         return cudaGetLastError();
     }
@@ -32,13 +35,23 @@ static cudaError_t launch_ex(void (*kern)(KArgs...), dim3 grid, dim3 block, cuda
     cfg.gridDim = grid;
     cfg.blockDim = block;
     cfg.stream = st;
-    cudaLaunchAttribute at[1];
-    at[0].id = cudaLaunchAttributeAccessPolicyWindow;
-    at[0].val.accessPolicyWindow = win->w;
+    cudaLaunchAttribute at[2];
+    unsigned na = 0;
+    if (w) {
+        at[na].id = cudaLaunchAttributeAccessPolicyWindow;
+        at[na++].val.accessPolicyWindow = win->w;
+    }
+    if (pdl) {
+        at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[na++].val.programmaticStreamSerializationAllowed = 1;
+    }
     cfg.attrs = at;
-    cfg.numAttrs = 1;
+    cfg.numAttrs = na;
     return cudaLaunchKernelEx(&cfg, kern, args...);
 }
+
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" :::); }
 
 __device__ __forceinline__ void append_count(unsigned long long* cnt)
 {
@@ -190,8 +203,9 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
     state<false, kClass0 ? 0 : -1>(O, r, t, p, v);
 #endif
     int c[3];
-    uint32_t next = kNil;
+    uint32_t next = kNil, ctag = 0;
     if (kChained && cell_of(g, p, c)) {
+        ctag = cell_tag(c[0], c[1], c[2]);
         // chained spatial hash: push onto the list of bucket hash(cell) -- one atomic exchange;
         // heads hold index + 1 (0 = empty bucket)
         const uint32_t b = chain_bucket(c[0], c[1], c[2], tab.bmask);
@@ -221,7 +235,7 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
     en.y = p[1];
     en.z = p[2];
     en.next = next;
-    en.pad = 0;
+    en.tag = ctag;
 #ifdef CD_STREAM_ENTRIES
     // written once here, read once (coalesced) by the next launch's scan: stream past L2 so the
     // randomly accessed slot table and bitmaps keep it
@@ -244,9 +258,10 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
 //      once, by the later-inserted object (no probe needed);
 //  (2) other cells: half-shell mode (L < 2 g_c, the paper's cell g_c) probes the 13
 //      positive half-shell neighbours -- each unordered pair of cells of a 3x3x3 block once;
-//      ball mode (L >= 2 g_c) probes the 0-7 other cells overlapping |x - p| < g_c -- a pair is
-//      seen from both objects and reported by the smaller index.  Each probe first tests the
-//      occupancy bitmap (all bitmap loads of a thread are issued together).
+//      ball mode (L >= 2 g_c) probes those of the 0-7 other cells overlapping |x - p| < g_c
+//      that lie in the positive (lexicographic) half-space of the own cell -- a pair in two
+//      cells is seen only from the smaller cell.  Each probe first tests the occupancy bitmap
+//      (all bitmap loads of a thread are issued together).
 // A pair is a candidate iff |r_i - r_j| < g_c (reading R6); candidates are appended with one
 // atomic per group of converged lanes (P:95 saves ids + sampling step).
 // ---------------------------------------------------------------------------------------
@@ -354,8 +369,11 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
         // (c +- 1 stays inside the 19-bit key range because |c| <= kCellMax = 2^18 - 2)
         const uint32_t hx1 = hx0 + (uint32_t)d0 * kHX, hy1 = hy0 + (uint32_t)d1 * kHY,
                        hz1 = hz0 + (uint32_t)d2 * kHZ;
-        // cell c + (b0 d0, b1 d1, b2 d2), b = 1..7, exists iff every axis set in b has d != 0
-        const uint32_t valid = (d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu) & 0xFEu;
+        // cell c + (b0 d0, b1 d1, b2 d2), b = 1..7, exists iff every axis set in b has d != 0;
+        // only cells in the positive lexicographic half-space of c are probed, so a pair in two
+        // cells is seen from exactly one of them (as in the half-shell scan)
+        const uint32_t pos = (d0 > 0 ? 0xAAu : 0u) | (d1 > 0 ? 0x44u : 0u) | (d2 > 0 ? 0x10u : 0u);
+        const uint32_t valid = (d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu) & pos;
         uint32_t hit = 0;
 #pragma unroll
         for (int b = 1; b < 8; ++b) {
@@ -367,7 +385,7 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
             const int b = __ffs(hit) - 1;
             hit &= hit - 1;
             probe_cell(g, slots, mask, tag, c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0),
-                       c[2] + ((b & 4) ? d2 : 0), E, (uint32_t)r, p, true, step, q, qcap, ctrl);
+                       c[2] + ((b & 4) ? d2 : 0), E, (uint32_t)r, p, false, step, q, qcap, ctrl);
         }
     }
 }
@@ -376,28 +394,53 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
 // bucket may also hold objects of other cells -- the exact distance test filters them.
 //  * pairs inside the object's own bucket (same cell, or a colliding cell) are found by the
 //    later-inserted object walking its own list successors (no probe);
-//  * every other bucket of its neighbourhood (own cell's 0-7 ball cells, or all 27 cells when
-//    L < 2 g_c), distinct and different from the own bucket, is walked in full and a pair is
-//    reported only from its smaller id -- for a pair closer than g_c in different buckets each
-//    object's neighbourhood contains the other's cell, so the smaller id sees it exactly once.
-__device__ __forceinline__ void walk_bucket(const GridGeom& g, const Entry* __restrict__ E,
-                                            uint32_t h, uint32_t epoch, uint32_t r, uint32_t my_next,
-                                            const double p[3], uint32_t step, Cand* __restrict__ q,
-                                            size_t qcap, Ctrl* ctrl)
+//  * ball mode (L >= 2 g_c): the buckets of the 0-7 ball cells in the positive half-space of
+//    the own cell are walked; only entries tagged with the probed cell count (walk_bucket_tag),
+//    so a pair in cells A != B is reported once, by the object whose cell is lexicographically
+//    smaller (parity hashing keeps these buckets distinct from each other and the own bucket);
+//  * half-shell mode (L < 2 g_c, rare with this table): all 26 neighbour buckets, de-duplicated,
+//    are walked in full and a pair is reported only from its smaller id (walk_bucket_gt).
+__device__ __forceinline__ uint32_t head_index(uint32_t h, uint32_t epoch)
 {
-    uint32_t j = ((h >> kEpochShift) == epoch && (h & kIdxMask)) ? (h & kIdxMask) - 1u : kNil;
+    return ((h >> kEpochShift) == epoch && (h & kIdxMask)) ? (h & kIdxMask) - 1u : kNil;
+}
+
+// half-shell mode (26 neighbour buckets, each walked in full): report from the smaller id
+__device__ __forceinline__ void walk_bucket_gt(const GridGeom& g, const Entry* __restrict__ E,
+                                               uint32_t h, uint32_t epoch, uint32_t r, const double p[3],
+                                               uint32_t step, Cand* __restrict__ q, size_t qcap,
+                                               Ctrl* ctrl)
+{
+    uint32_t j = head_index(h, epoch);
     uint32_t guard = g.max_walk;
     while (j != kNil) {
         if (guard-- == 0) {
             ctrl->err_internal = 1;
             return;
         }
-        if (j == r) {
-            j = my_next;
-            continue;
-        }
         const Entry ej = E[j];
         if (j > r) test_pair(g, r, j, p, ej, step, q, qcap, ctrl);
+        j = ej.next;
+    }
+}
+
+// ball mode: bucket of the probed cell (tag ctag), which lies in the positive half-space of the
+// scanning object's cell -- only the probed cell's own entries count (a colliding neighbour
+// cell's entries are found by their own probe, so each pair is reported exactly once)
+__device__ __forceinline__ void walk_bucket_tag(const GridGeom& g, const Entry* __restrict__ E,
+                                                uint32_t h, uint32_t epoch, uint32_t ctag, uint32_t r,
+                                                const double p[3], uint32_t step,
+                                                Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
+{
+    uint32_t j = head_index(h, epoch);
+    uint32_t guard = g.max_walk;
+    while (j != kNil) {
+        if (guard-- == 0) {
+            ctrl->err_internal = 1;
+            return;
+        }
+        const Entry ej = E[j];
+        if (ej.tag == ctag) test_pair(g, r, j, p, ej, step, q, qcap, ctrl);
         j = ej.next;
     }
 }
@@ -431,14 +474,19 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
                     if (!dup) bk[nb++] = b;
                 }
         for (int k = 0; k < nb; ++k)
-            walk_bucket(g, E, __ldg(heads + bk[k]), epoch, (uint32_t)r, me.next, p, step, q, qcap, ctrl);
+            walk_bucket_gt(g, E, __ldg(heads + bk[k]), epoch, (uint32_t)r, p, step, q, qcap, ctrl);
         return;
     }
     const double rl = g.reach * g.inv_cell;
     const int d0 = fr[0] < rl ? -1 : (fr[0] > 1.0 - rl ? 1 : 0);
     const int d1 = fr[1] < rl ? -1 : (fr[1] > 1.0 - rl ? 1 : 0);
     const int d2 = fr[2] < rl ? -1 : (fr[2] > 1.0 - rl ? 1 : 0);
-    const uint32_t valid = (d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu) & 0xFEu;
+    // ball cells (offset o_b = (b&1 ? d0 : 0, b&2 ? d1 : 0, b&4 ? d2 : 0)) in the positive
+    // lexicographic half-space o > 0 only: a pair in cells A != B is then probed from exactly
+    // one side (B - A > 0 or A - B > 0), and B is in the ball set of the object in A whenever
+    // the pair is closer than g_c
+    const uint32_t pos = (d0 > 0 ? 0xAAu : 0u) | (d1 > 0 ? 0x44u : 0u) | (d2 > 0 ? 0x10u : 0u);
+    const uint32_t valid = (d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu) & pos;
     if (!valid) return;
     // the ball's cells differ pairwise in parity -> distinct buckets, no de-duplication
     uint32_t hd[8];
@@ -450,7 +498,11 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
                     : 0u;
 #pragma unroll
     for (int b = 1; b < 8; ++b)
-        if (hd[b]) walk_bucket(g, E, hd[b], epoch, (uint32_t)r, me.next, p, step, q, qcap, ctrl);
+        if (hd[b])
+            walk_bucket_tag(g, E, hd[b], epoch,
+                            cell_tag(c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0),
+                                     c[2] + ((b & 4) ? d2 : 0)),
+                            (uint32_t)r, p, step, q, qcap, ctrl);
 }
 
 // ---------------------------------------------------------------------------------------
@@ -473,6 +525,12 @@ __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
 #ifdef CD_ABL_NO_BUILD
     if (bx < nA + nB) return;
 #endif
+    // Programmatic dependent launch (chained grid, StepArgs::pdl): build blocks depend on no
+    // earlier launch still running -- the head/entry sets they write were last read two launches
+    // ago, and this launch started only after every block of the previous one had triggered,
+    // which its scan blocks do after their own wait -- so they trigger at once.  Scan blocks
+    // read the previous launch's build output: wait for its completion, then trigger.
+    if (bx < nA + nB) pdl_trigger();
     if (bx < nA) {
         const int s = (int)(bx / nbA);
         const int64_t r = (int64_t)(bx % nbA) * 256 + threadIdx.x;
@@ -488,6 +546,8 @@ __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
                                       a.dt, a.build_tag, a.ctrl);
     } else {
         const uint32_t b3 = bx - nA - nB;
+        pdl_wait();
+        pdl_trigger();
         // zero the bitmap set of batch b + 2 (all Bmax tables), grid-stride over role-C threads
         const int64_t tid = (int64_t)b3 * 256 + threadIdx.x;
         const int64_t nth = a.nCblocks * 256;
@@ -522,8 +582,8 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
     const int64_t blocks = a.build_B * (a.nbA + a.nbB) + a.nCblocks;
     if (blocks == 0) return cudaSuccess;
     lc.bump();
-    if (a.chained) return launch_ex(k_step<true>, dim3((unsigned)blocks), dim3(256), st, win, a);
-    return launch_ex(k_step<false>, dim3((unsigned)blocks), dim3(256), st, win, a);
+    if (a.chained) return launch_ex(k_step<true>, dim3((unsigned)blocks), dim3(256), st, win, a.pdl != 0, a);
+    return launch_ex(k_step<false>, dim3((unsigned)blocks), dim3(256), st, win, false, a);
 }
 
 // ---------------------------------------------------------------------------------------
