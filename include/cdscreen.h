@@ -173,6 +173,10 @@ cd_status cd_propagate(const cd_elements* el, size_t n, const double* t, size_t 
  * an all-gather.  Requires i < j in every record. */
 cd_status cd_conjunctions_sort_device(cd_conjunction* data, size_t n, void* stream);
 
+/* Release a result of cd_screen / cd_screen_ex.  Host results are freed immediately.  Device
+ * results (outputs_on_device) are released stream-ordered (cudaFreeAsync) on the stream the call
+ * ran on (cd_options.stream, or the legacy default stream when the library used its own), so
+ * work the caller queued on that stream may still read them; no device-wide synchronisation. */
 void cd_conjunctions_free(cd_conjunctions* c);
 void cd_candidates_free(cd_candidate* c);
 const char* cd_status_str(cd_status s);

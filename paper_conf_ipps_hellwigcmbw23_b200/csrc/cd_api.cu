@@ -106,6 +106,32 @@ struct DBuf {
 std::mutex g_pool_mu;
 bool g_pool_done[64] = {};
 
+// Per-host-thread page-locked staging for the per-round counters (4 Ctrl-sized slots), allocated
+// once and kept for the thread's lifetime: no call pays cudaMallocHost / cudaFreeHost.
+struct PinnedStage {
+    Ctrl* p = nullptr;
+    ~PinnedStage()
+    {
+        if (p) cudaFreeHost(p);   // at thread exit (errors after context teardown are ignored)
+    }
+};
+thread_local PinnedStage g_stage;
+
+cd_status pinned_stage(Ctrl** out)
+{
+    if (!g_stage.p) {
+        void* p = nullptr;
+        if (cudaMallocHost(&p, 4 * sizeof(Ctrl)) != cudaSuccess || !p)
+            return fail(CD_ENOMEM, "page-locked staging allocation failed");
+        g_stage.p = static_cast<Ctrl*>(p);
+    }
+    *out = g_stage.p;
+    return CD_OK;
+}
+
+// Compute capability per device, queried once (cudaGetDeviceProperties costs milliseconds).
+int g_cc[64];   // 0 = not yet queried, else major * 10 + minor
+
 void setup_pool(int dev)
 {
     std::lock_guard<std::mutex> lk(g_pool_mu);
@@ -121,6 +147,7 @@ void setup_pool(int dev)
 struct Owner {
     bool device;
     void* p;
+    cudaStream_t st;   // device results: released stream-ordered on the call's stream
 };
 
 // Optional per-phase device timing (cd_options.profile_phases): CUDA events recorded on the
@@ -191,13 +218,20 @@ struct PhaseTimer {
     void harvest()
     {
         if (!on) return;
+        // marks of a round still in flight (pipelined rounds) stay for a later harvest
+        std::vector<Mark> keep;
         for (const Mark& m : marks) {
+            if (cudaEventQuery(pool[m.b]) != cudaSuccess) {
+                keep.push_back(m);
+                continue;
+            }
             float x = 0.f;
             if (cudaEventElapsedTime(&x, pool[m.a], pool[m.b]) == cudaSuccess) ms[m.ph] += x;
             launches[m.ph] += m.nl;
         }
-        marks.clear();
-        used = 0;
+        cudaGetLastError();   // clear cudaErrorNotReady
+        marks.swap(keep);
+        if (marks.empty() && cur < 0) used = 0;
     }
     void to_stats(cd_stats& s) const
     {
@@ -244,11 +278,17 @@ struct Call {
         dev = o.device >= 0 ? o.device : prev_dev;
         if (dev >= ndev) return fail(CD_EINVAL, "device %d out of range (%d devices)", dev, ndev);
         CU(cudaSetDevice(dev));
-        cudaDeviceProp prop;
-        CU(cudaGetDeviceProperties(&prop, dev));
-        if (prop.major != 10 || prop.minor != 0)
-            return fail(CD_ENODEV, "libcdscreen is built for sm_100a (B200); device %d is sm_%d%d",
-                        dev, prop.major, prop.minor);
+        int cc = dev < 64 ? g_cc[dev] : 0;
+        if (!cc) {
+            int major = 0, minor = 0;
+            CU(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev));
+            CU(cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev));
+            cc = 10 * major + minor;
+            if (dev < 64) g_cc[dev] = cc;
+        }
+        if (cc != 100)
+            return fail(CD_ENODEV, "libcdscreen is built for sm_100a (B200); device %d is sm_%d",
+                        dev, cc);
         setup_pool(dev);
         if (o.stream) {
             st = (cudaStream_t)o.stream;
@@ -546,75 +586,94 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     CU(cudaMemsetAsync(ctrl.p, 0, sizeof(Ctrl), st));
     DBuf<unsigned long long> nwork(st);
     CU(nwork.alloc(1));
-    Ctrl* hctrl = nullptr;
-    DBG("run: queues allocated");
-    CU(cudaMallocHost((void**)&hctrl, sizeof(Ctrl) + sizeof(unsigned long long)));
-    DBG("run: pinned ctrl");
-    struct HostFree {
-        void* p;
-        ~HostFree() { cudaFreeHost(p); }
-    } hf{hctrl};
-    unsigned long long* hnwork = reinterpret_cast<unsigned long long*>(hctrl + 1);
+    // pinned host staging of the per-round counters: two slots (rounds r and r + 1 in flight),
+    // cached per host thread so no call pays a page-locked allocation (an RM call that contends
+    // with NVML clients such as nvidia-smi)
+    Ctrl* hslot[2];
+    unsigned long long* hnw[2];
+    {
+        Ctrl* base = nullptr;
+        TRY(pinned_stage(&base));
+        for (int s = 0; s < 2; ++s) {
+            hslot[s] = base + 2 * s;
+            hnw[s] = reinterpret_cast<unsigned long long*>(base + 2 * s + 1);
+        }
+    }
+    DBG("run: staging ready");
+    cudaEvent_t rev[2] = {nullptr, nullptr};
+    struct EvFree {
+        cudaEvent_t* e;
+        ~EvFree() { for (int s = 0; s < 2; ++s) if (e[s]) cudaEventDestroy(e[s]); }
+    } evf{rev};
+    for (int s = 0; s < 2; ++s) CU(cudaEventCreateWithFlags(&rev[s], cudaEventDisableTiming));
 
     int64_t Rsteps = o.round_steps ? (int64_t)o.round_steps
                                    : std::max<int64_t>(1, (int64_t)(qcap / 2 / (size_t)std::max<int64_t>(1, n / 20)));
+    // cumulative device counters as of the last accepted round (the rollback state of a redo)
     unsigned long long conj_before = 0;
     unsigned long long hyb_before[4] = {0, 0, 0, 0};
-    int64_t k = kb;
-    while (k < ke) {
-        const int64_t Rk = std::min<int64_t>(Rsteps, ke - k);
+    // the cell edge is settled once the first round has measured the candidate density
+    bool settled = !auto_cell;
+    // rounds are software-pipelined one deep: round r + 1 is enqueued before the host waits for
+    // round r's counters, so the GPU never idles while the host checks capacities and enqueues
+    // the next ~500 launches.  Capacity overflows are rare: the later round is drained and both
+    // are redone.  The candidate hook (Want::Cand) copies each accepted round's queue out, so it
+    // runs unpipelined.
+    const int depth = want == Want::Cand ? 1 : 2;
+    struct Round { int64_t k, Rk; int slot; size_t qcap; };   // qcap: the capacity it ran with
+    Round inflight[2];
+    int nin = 0, next_slot = 0;
+    auto enqueue_round = [&](int64_t kr, int64_t Rk, int slot) -> cd_status {
         CU(cudaMemsetAsync(&ctrl.p->n_cand, 0, sizeof(unsigned long long), st));
         CU(cudaMemsetAsync(nwork.p, 0, sizeof(unsigned long long), st));
-        {
-            // software pipeline over the round's batches: launch i builds batch i and scans i - 1
-            const int64_t J = (Rk + Bmax - 1) / Bmax;
-            for (int64_t i = 0; i <= J; ++i) {
-                StepArgs sa{};
-                sa.O = O;
-                sa.g = g;
-                sa.mask = mask;
-                sa.t0 = t0;
-                sa.dt = dt;
-                sa.q = q.p;
-                sa.qcap = qcap;
-                sa.ctrl = ctrl.p;
-                const uint64_t bb = batch_no + (uint64_t)i;   // batch built in this launch
-                if (i < J) {
-                    if (chained && bb % 255u < 3 && bb >= 3) {
-                        // head set bb % 3 is used by batches of one residue mod 3; its epochs
-                        // (bb % 255 + 1) would repeat within the next 255 batches: zero it (its
-                        // last scan, of batch bb - 3, finished two launches ago)
-                        CU(cudaMemsetAsync(bitset[bb % 3], 0, bit_bytes, st));
-                    }
-                    if (can_open && bb % kMaxTag < 2 && bb >= 2) {
-                        // this slot set's tags wrap with this batch: zero it (its last scan, of
-                        // batch bb - 2, finished in the previous launch)
-                        CU(cudaMemsetAsync(slotset[bb % 2], 0, slot_bytes, st));
-                    }
-                    sa.build_k0 = k + i * Bmax;
-                    sa.build_B = std::min<int64_t>(Bmax, k + Rk - sa.build_k0);
-                    sa.build_tab = tab_of(bb);
-                    sa.build_ents = entbuf[bb % 3];
-                    sa.build_tag = tag_of(bb);
+        // software pipeline over the round's batches: launch i builds batch i and scans i - 1
+        const int64_t J = (Rk + Bmax - 1) / Bmax;
+        for (int64_t i = 0; i <= J; ++i) {
+            StepArgs sa{};
+            sa.O = O;
+            sa.g = g;
+            sa.mask = mask;
+            sa.t0 = t0;
+            sa.dt = dt;
+            sa.q = q.p;
+            sa.qcap = qcap;
+            sa.ctrl = ctrl.p;
+            const uint64_t bb = batch_no + (uint64_t)i;   // batch built in this launch
+            if (i < J) {
+                if (chained && bb % 255u < 3 && bb >= 3) {
+                    // head set bb % 3 is used by batches of one residue mod 3; its epochs
+                    // (bb % 255 + 1) would repeat within the next 255 batches: zero it (its
+                    // last scan, of batch bb - 3, finished two launches ago)
+                    CU(cudaMemsetAsync(bitset[bb % 3], 0, bit_bytes, st));
                 }
-                if (i > 0) {
-                    sa.scan_k0 = k + (i - 1) * Bmax;
-                    sa.scan_B = std::min<int64_t>(Bmax, k + Rk - sa.scan_k0);
-                    sa.scan_tab = tab_of(bb - 1);
-                    sa.scan_ents = entbuf[(bb - 1) % 3];
-                    sa.scan_tag = tag_of(bb - 1);
+                if (can_open && bb % kMaxTag < 2 && bb >= 2) {
+                    // this slot set's tags wrap with this batch: zero it (its last scan, of
+                    // batch bb - 2, finished in the previous launch)
+                    CU(cudaMemsetAsync(slotset[bb % 2], 0, slot_bytes, st));
                 }
-                sa.zero_bits = bitset[(bb + 1) % 3];   // batch bb - 2's bitmaps, next built by bb + 1
-                sa.zero_bits_words = bwords;
-                sa.zero_depth = chained ? 0 : Bmax;   // chained heads are epoch-tagged
-                sa.chained = chained ? 1 : 0;
-                sa.pdl = chained && !no_pdl ? 1 : 0;
-                if (i == 0) C.pt.span_start(kPhScan);
-                CU(launch_step(sa, &win, st, C.lc));
+                sa.build_k0 = kr + i * Bmax;
+                sa.build_B = std::min<int64_t>(Bmax, kr + Rk - sa.build_k0);
+                sa.build_tab = tab_of(bb);
+                sa.build_ents = entbuf[bb % 3];
+                sa.build_tag = tag_of(bb);
             }
-            C.pt.span_stop((uint64_t)J + 1);
-            batch_no += (uint64_t)J;
+            if (i > 0) {
+                sa.scan_k0 = kr + (i - 1) * Bmax;
+                sa.scan_B = std::min<int64_t>(Bmax, kr + Rk - sa.scan_k0);
+                sa.scan_tab = tab_of(bb - 1);
+                sa.scan_ents = entbuf[(bb - 1) % 3];
+                sa.scan_tag = tag_of(bb - 1);
+            }
+            sa.zero_bits = bitset[(bb + 1) % 3];   // batch bb - 2's bitmaps, next built by bb + 1
+            sa.zero_bits_words = bwords;
+            sa.zero_depth = chained ? 0 : Bmax;   // chained heads are epoch-tagged
+            sa.chained = chained ? 1 : 0;
+            sa.pdl = chained && !no_pdl ? 1 : 0;
+            if (i == 0) C.pt.span_start(kPhScan);
+            CU(launch_step(sa, &win, st, C.lc));
         }
+        C.pt.span_stop((uint64_t)J + 1);
+        batch_no += (uint64_t)J;
         if (want == Want::Conj) {
             C.pt.start(kPhRefine);
             if (mode == CD_HYBRID) {
@@ -628,23 +687,44 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             }
             C.pt.stop();
         }
-        CU(cudaMemcpyAsync(hctrl, ctrl.p, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
-        CU(cudaMemcpyAsync(hnwork, nwork.p, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
-        DBG("round: enqueued", (long long)k, (long long)Rk);
-        CU(cudaStreamSynchronize(st));
-        DBG("round: synced", (long long)k, (long long)Rk);
+        CU(cudaMemcpyAsync(hslot[slot], ctrl.p, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
+        CU(cudaMemcpyAsync(hnw[slot], nwork.p, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+        CU(cudaEventRecord(rev[slot], st));
+        DBG("round: enqueued", (long long)kr, (long long)Rk);
+        return CD_OK;
+    };
+
+    int64_t k = kb;
+    while (k < ke || nin > 0) {
+        if (k < ke && nin < depth && (settled || nin == 0)) {
+            const int64_t Rk = std::min<int64_t>(Rsteps, ke - k);
+            const int slot = next_slot;
+            next_slot ^= 1;
+            TRY(enqueue_round(k, Rk, slot));
+            inflight[nin++] = Round{k, Rk, slot, qcap};
+            k += Rk;
+            continue;
+        }
+        // wait for the oldest round in flight
+        const Round rd = inflight[0];
+        if (nin == 2) inflight[0] = inflight[1];
+        --nin;
+        CU(cudaEventSynchronize(rev[rd.slot]));
+        DBG("round: synced", (long long)rd.k, (long long)rd.Rk);
         C.pt.harvest();
+        const Ctrl* hctrl = hslot[rd.slot];
+        const unsigned long long hnwork = *hnw[rd.slot];
         if (hctrl->err_internal)
             return fail(CD_EINTERNAL, "internal: a grid cell list did not terminate");
         if (hctrl->err_range)
             return fail(CD_ERANGE, "a position fell outside the cell-key range (+-%lld cells of %g km)",
                         (long long)kCellMax, L);
         bool redo = false;
-        if (hctrl->n_cand > qcap) {
+        if (hctrl->n_cand > rd.qcap) {
             ++stats.retries;
-            if (Rk > 1) {
-                const double rate = (double)hctrl->n_cand / (double)Rk;
-                Rsteps = std::max<int64_t>(1, std::min<int64_t>(Rk / 2, (int64_t)(0.5 * qcap / rate)));
+            if (rd.Rk > 1) {
+                const double rate = (double)hctrl->n_cand / (double)rd.Rk;
+                Rsteps = std::max<int64_t>(1, std::min<int64_t>(rd.Rk / 2, (int64_t)(0.5 * rd.qcap / rate)));
             } else {
                 qcap = (size_t)(hctrl->n_cand * 1.25) + 1024;
                 CU(q.alloc(qcap));
@@ -654,9 +734,9 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                 }
             }
             redo = true;
-        } else if (want == Want::Conj && *hnwork > wcap) {
+        } else if (want == Want::Conj && hnwork > wcap) {
             ++stats.retries;
-            wcap = (size_t)(*hnwork * 1.25) + 1024;
+            wcap = (size_t)(hnwork * 1.25) + 1024;
             CU(w.alloc(wcap));
             redo = true;
         } else if (want == Want::Conj && hctrl->n_conj > ocap) {
@@ -672,7 +752,11 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             redo = true;
         }
         if (redo) {
-            // roll the cumulative counters back to the start of the round
+            // drain the later round (if any), roll the cumulative counters back to the last
+            // accepted round and restart from this round's first step
+            CU(cudaStreamSynchronize(st));
+            C.pt.harvest();
+            nin = 0;
             Ctrl back = *hctrl;
             back.n_conj = conj_before;
             back.n_ap = hyb_before[0];
@@ -680,14 +764,18 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             back.n_path = hyb_before[2];
             back.n_time = hyb_before[3];
             back.n_cand = 0;
-            *hctrl = back;
-            CU(cudaMemcpyAsync(ctrl.p, hctrl, sizeof(Ctrl), cudaMemcpyHostToDevice, st));
+            back.err_range = 0;
+            back.err_internal = 0;
+            Ctrl* stage = hslot[rd.slot];
+            *stage = back;
+            CU(cudaMemcpyAsync(ctrl.p, stage, sizeof(Ctrl), cudaMemcpyHostToDevice, st));
             CU(cudaStreamSynchronize(st));
+            k = rd.k;
             continue;
         }
         // round accepted
         stats.candidates += hctrl->n_cand;
-        stats.refined += *hnwork;
+        stats.refined += hnwork;
         if (want == Want::Cand && hctrl->n_cand) {
             if (R.n_cand + hctrl->n_cand > ccap) {
                 const size_t ncap = std::max<size_t>(2 * ccap, R.n_cand + hctrl->n_cand + 1024);
@@ -708,18 +796,20 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         hyb_before[1] = hctrl->n_coplanar;
         hyb_before[2] = hctrl->n_path;
         hyb_before[3] = hctrl->n_time;
-        if (auto_cell && k == kb) {   // first round done: re-pick the cell edge from the density
-            const double m = choose_cell_factor((double)hctrl->n_cand / ((double)Rk * (double)n));
+        if (!settled) {   // first round done: pick the cell edge from the measured density
+            const double m = choose_cell_factor((double)hctrl->n_cand / ((double)rd.Rk * (double)n));
             L = gc * m;
             if (L < gc * (1.0 + 1e-12)) L = gc * (1.0 + 1e-12);
             g.inv_cell = 1.0 / L;
             g.halfshell = L < 2.0 * gc ? 1 : 0;
             chained = pick_chained(g);
+            settled = true;
         }
         if (!o.round_steps) {
-            const double rate = std::max(1.0, (double)hctrl->n_cand / (double)Rk);
-            // dense candidate rates (hybrid): grow the queue so a round spans >= 64 steps (each
-            // round ends with a host sync), within a 2^28-entry (3 GB) cap
+            const double rate = std::max(1.0, (double)hctrl->n_cand / (double)rd.Rk);
+            // dense candidate rates (hybrid): grow the queue so a round spans >= 64 steps, within
+            // a 2^28-entry (3 GB) cap.  The queue is reallocated stream-ordered: a round still
+            // in flight keeps the old buffer until it finishes.
             const double wanted = rate * 64.0 * 1.25;
             if (wanted > (double)qcap && qcap < (size_t(1) << 28)) {
                 qcap = (size_t)std::min(wanted, (double)(size_t(1) << 28));
@@ -727,13 +817,12 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             }
             Rsteps = std::max<int64_t>(1, std::min<int64_t>(1 << 16, (int64_t)(0.5 * qcap / rate)));
         }
-        k += Rk;
     }
     R.n_conj = (size_t)conj_before;
-    stats.hybrid_ap_rejected = hctrl->n_ap;
-    stats.hybrid_coplanar = hctrl->n_coplanar;
-    stats.hybrid_path_rejected = hctrl->n_path;
-    stats.hybrid_time_rejected = hctrl->n_time;
+    stats.hybrid_ap_rejected = hyb_before[0];
+    stats.hybrid_coplanar = hyb_before[1];
+    stats.hybrid_path_rejected = hyb_before[2];
+    stats.hybrid_time_rejected = hyb_before[3];
     return CD_OK;
 }
 
@@ -779,7 +868,7 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
             C.pt.stop();
         }
     }
-    Owner* own = new Owner{o.outputs_on_device != 0, nullptr};
+    Owner* own = new Owner{o.outputs_on_device != 0, nullptr, C.own_stream ? nullptr : C.st};
     if (R.n_conj) {
         if (o.outputs_on_device) {
             own->p = sorted.detach();
@@ -952,7 +1041,10 @@ void cd_conjunctions_free(cd_conjunctions* c)
     Owner* own = static_cast<Owner*>(c->_owner);
     if (own) {
         if (own->p) {
-            if (own->device) cudaFree(own->p);
+            // stream-ordered release (no device-wide synchronisation): after the work the
+            // caller queued on the call's stream (the legacy default stream if the library
+            // created its own)
+            if (own->device) cudaFreeAsync(own->p, own->st);
             else free(own->p);
         }
         delete own;
