@@ -178,6 +178,33 @@ cd_status cd_conjunctions_sort_device(cd_conjunction* data, size_t n, void* stre
  * ran on (cd_options.stream, or the legacy default stream when the library used its own), so
  * work the caller queued on that stream may still read them; no device-wide synchronisation. */
 void cd_conjunctions_free(cd_conjunctions* c);
+
+/* A-priori sizing of a screen (Section IV-B), pure host arithmetic: the
+ * paper's Extra-P candidate models and its memory-bounded grid count, evaluated for this
+ * library's data structures.  The library uses est_candidates_per_step to size a call's first
+ * round (queue capacity, probe length, initial cell edge) before any density is measured. */
+typedef struct {
+    double samples;                 /* o = K = floor((t1 - t0)/dt) + 1 sampling steps (R4)   */
+    double est_candidates;          /* c' over [t0, t1]: Eq. 3 (grid) 2.32e-9 n^2 s^(4/3) t d^(7/4),
+                                       Eq. 4 (hybrid) 2.14e-9 n^2 s^(5/3) t d; s = dt [s],
+                                       t = t1 - t0 [s] (dt if 0), d [km]                 */
+    double est_candidates_per_step; /* c' with t = dt                                                */
+    double capacity;                /* c = max(c', 10^4) * 2 * 2                             */
+    double capacity_bytes;          /* g_ch = c * 16 B                                       */
+    double fixed_bytes;             /* a_s + a_k + a_ch of this library: elements (48 B/object),
+                                       orbit records (325 B/object), first-round candidate queue
+                                       (12 B/entry) and work items (24 B/entry)                      */
+    double bytes_per_grid;          /* a_gh + a_l: one step's grid table + 32 B entries per object   */
+    double grids_in_memory;         /* p = (m - a_s - a_k - a_ch) / (a_gh + a_l)             */
+    double rounds;                  /* r_c = o / p; +inf if p = 0                            */
+    double cell_factor;             /* the auto cell edge L / g_c for the a-priori density           */
+} cd_plan_info;
+
+/* Fill *out for screening n objects over [t0, t1] at step dt, threshold d, in mode, with
+ * mem_bytes of free device memory m (0 = query the current device: CD_ENODEV without one).
+ * Validation as cd_screen (CD_EINVAL); out must be non-NULL. */
+cd_status cd_plan(size_t n, double t0, double t1, double dt, double d, cd_mode mode,
+                  size_t mem_bytes, cd_plan_info* out);
 void cd_candidates_free(cd_candidate* c);
 const char* cd_status_str(cd_status s);
 const char* cd_last_error(void);

@@ -31,7 +31,7 @@ CAND_DTYPE = np.dtype([("i", "<u4"), ("j", "<u4"), ("step", "<u4")])
 # C ABI symbols declared in include/cdscreen.h
 ABI_SYMBOLS = ("cd_options_init", "cd_screen", "cd_screen_ex", "cd_candidates", "cd_propagate",
                "cd_conjunctions_sort_device", "cd_conjunctions_free", "cd_candidates_free", "cd_status_str", "cd_last_error",
-               "cd_abi_version", "cd_kernel_launches")
+               "cd_abi_version", "cd_kernel_launches", "cd_plan")
 
 
 class CdError(RuntimeError):
@@ -85,6 +85,15 @@ class cd_options(C.Structure):
                 ("stats", C.POINTER(cd_stats))]
 
 
+class cd_plan_info(C.Structure):
+    _fields_ = [(k, C.c_double) for k in (
+        "samples", "est_candidates", "est_candidates_per_step", "capacity", "capacity_bytes",
+        "fixed_bytes", "bytes_per_grid", "grids_in_memory", "rounds", "cell_factor")]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
 _lib = None
 
 
@@ -123,6 +132,9 @@ def lib():
         L.cd_last_error.restype = C.c_char_p
         L.cd_abi_version.restype = C.c_int
         L.cd_kernel_launches.restype = C.c_uint64
+        L.cd_plan.restype = C.c_int
+        L.cd_plan.argtypes = [C.c_size_t, C.c_double, C.c_double, C.c_double, C.c_double, C.c_int,
+                              C.c_size_t, P(cd_plan_info)]
         _lib = L
     return _lib
 
@@ -183,6 +195,10 @@ def cd_abi_version() -> int:
 
 def cd_kernel_launches() -> int:
     return int(lib().cd_kernel_launches())
+
+
+def cd_plan(n, t0, t1, dt, d, mode, mem_bytes, out):
+    return lib().cd_plan(n, t0, t1, dt, d, mode, mem_bytes, C.byref(out))
 
 
 # numpy / torch wrappers --------------------------------------------------------------------
@@ -307,3 +323,10 @@ def propagate(pop, times, velocity=False, **kw):
                         v.ctypes.data if velocity else None, opt))
     return (xyz, v) if velocity else xyz
 
+
+
+def plan(n, t0, t1, dt, d, mode="grid", mem_bytes=0):
+    """A-priori sizing (Extra-P candidate model, grids in memory, rounds) as a dict."""
+    out = cd_plan_info()
+    _check(cd_plan(int(n), float(t0), float(t1), float(dt), float(d), _mode(mode), int(mem_bytes), out))
+    return out.as_dict()

@@ -450,6 +450,28 @@ double choose_cell_factor(double c)
     return best;
 }
 
+// A-priori candidate count, the paper's Extra-P models (Section IV-B):
+//   grid   (Eq. 3)  c' = 2.32e-9 n^2 s^(4/3) t d^(7/4)
+//   hybrid (Eq. 4)  c' = 2.14e-9 n^2 s^(5/3) t d
+// n objects, s seconds per sample, t simulated span [s], d threshold [km].  c' counts the
+// (ids, step) entries of the paper's conjunction hash map, i.e. the candidate set; on the
+// paper-shaped config-4 population it lands within 2x of the measured count.
+double extra_p_candidates(double n, double s, double t, double d, cd_mode mode)
+{
+    if (mode == CD_HYBRID) return 2.14e-9 * n * n * std::pow(s, 5.0 / 3.0) * t * d;
+    return 2.32e-9 * n * n * std::pow(s, 4.0 / 3.0) * t * std::pow(d, 1.75);
+}
+
+// Initial candidate-queue capacity (entries) of one call: at least 4M and 4n, grown so that a
+// round at the a-priori candidate rate spans >= 64 steps (2^28 cap), like the measured-rate rule
+size_t initial_qcap(int64_t n, double est_step)
+{
+    size_t qcap = std::max<size_t>(size_t(1) << 22, 4 * (size_t)n);
+    const double wanted = est_step * 64.0 * 1.25;
+    if (wanted > (double)qcap) qcap = (size_t)std::min(wanted, (double)(size_t(1) << 28));
+    return qcap;
+}
+
 struct Result {
     DBuf<Conj> conj;        // unsorted conjunction records (internal ids)
     size_t n_conj = 0;
@@ -469,10 +491,13 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     stats.steps = (uint64_t)(ke - kb);
     stats.object_steps = (uint64_t)(ke - kb) * (uint64_t)n;
     const double gc = d + o.v_margin * dt;   // Eq. 1
-    // grid cell edge L = m g_c (m = cell_factor; 0 = auto: start at 4, then choose from the
-    // candidate density measured in the first round, see choose_cell_factor)
+    // grid cell edge L = m g_c (m = cell_factor; 0 = auto: start from the a-priori density, then
+    // choose from the candidate density measured in the first round, see choose_cell_factor)
     const bool auto_cell = o.cell_factor == 0.0;
-    double L = gc * (auto_cell ? 4.0 : o.cell_factor);
+    // a-priori candidates per step (Eq. 3 / Eq. 4 with t = one sample): sizes the first round
+    // and seeds the auto cell edge before the first round measures the real density
+    const double est_step = std::max(1.0, extra_p_candidates((double)n, dt, dt, d, mode));
+    double L = gc * (auto_cell ? choose_cell_factor(est_step / std::max<double>(1.0, (double)n)) : o.cell_factor);
     if (L < gc * (1.0 + 1e-12)) L = gc * (1.0 + 1e-12);
     GridGeom g;
     g.ox = o.grid_origin[0];
@@ -564,10 +589,12 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         }
         cudaGetLastError();   // persistence is best effort
     }
-    size_t qcap = std::max<size_t>(size_t(1) << 22, 4 * (size_t)n);
+    size_t qcap = initial_qcap(n, est_step);
     DBuf<Cand> q(st);
     CU(q.alloc(qcap));
-    size_t wcap = want == Want::Conj ? qcap : 0;
+    // work items (prefilter / hybrid-filter survivors) are a small fraction of the candidates:
+    // start at the base capacity, grow on demand (retry path)
+    size_t wcap = want == Want::Conj ? std::min(qcap, std::max<size_t>(size_t(1) << 22, 4 * (size_t)n)) : 0;
     DBuf<Work> w(st);
     if (want == Want::Conj) CU(w.alloc(wcap));
     size_t ocap = size_t(1) << 20;
@@ -607,8 +634,12 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     } evf{rev};
     for (int s = 0; s < 2; ++s) CU(cudaEventCreateWithFlags(&rev[s], cudaEventDisableTiming));
 
+    // first round: half the queue at the a-priori rate; in auto-cell mode it is also the density
+    // probe, kept short (enough candidates for a density estimate, <= 41 steps)
     int64_t Rsteps = o.round_steps ? (int64_t)o.round_steps
-                                   : std::max<int64_t>(1, (int64_t)(qcap / 2 / (size_t)std::max<int64_t>(1, n / 20)));
+                                   : std::max<int64_t>(1, std::min<int64_t>(1 << 16, (int64_t)(0.5 * (double)qcap / est_step)));
+    if (!o.round_steps && auto_cell)
+        Rsteps = std::max<int64_t>(1, std::min<int64_t>(Rsteps, std::min<int64_t>(41, (int64_t)std::ceil(2e5 / est_step))));
     // cumulative device counters as of the last accepted round (the rollback state of a redo)
     unsigned long long conj_before = 0;
     unsigned long long hyb_before[4] = {0, 0, 0, 0};
@@ -1052,6 +1083,56 @@ void cd_conjunctions_free(cd_conjunctions* c)
     c->data = nullptr;
     c->count = 0;
     c->_owner = nullptr;
+}
+
+cd_status cd_plan(size_t n, double t0, double t1, double dt, double d, cd_mode mode,
+                  size_t mem_bytes, cd_plan_info* out)
+{
+    try {
+        if (!out) return fail(CD_EINVAL, "out must be non-NULL");
+        memset(out, 0, sizeof *out);
+        if (mode != CD_GRID && mode != CD_HYBRID) return fail(CD_EINVAL, "unknown mode %d", (int)mode);
+        cd_options o;
+        cd_options_init(&o);
+        int64_t K = 0;
+        TRY(validate_scalars(n, t0, t1, dt, d, o, &K));
+        if (mem_bytes == 0) {
+            int ndev = 0;
+            if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+                return fail(CD_ENODEV, "mem_bytes = 0 needs a CUDA device (free memory query)");
+            size_t fr = 0, tot = 0;
+            CU(cudaMemGetInfo(&fr, &tot));
+            mem_bytes = fr;
+        }
+        const double nn = (double)n;
+        const double span = t1 - t0 > 0.0 ? t1 - t0 : dt;
+        out->samples = (double)K;
+        out->est_candidates = extra_p_candidates(nn, dt, span, d, mode);
+        out->est_candidates_per_step = extra_p_candidates(nn, dt, dt, d, mode);
+        out->capacity = std::max(out->est_candidates, 1e4) * 2.0 * 2.0;
+        out->capacity_bytes = out->capacity * 16.0;
+        // this library's structures: a_s elements, a_k orbit records + class +
+        // permutation, a_ch the round's candidate queue (12 B) and work items (24 B)
+        const double qcap = (double)initial_qcap((int64_t)n, std::max(1.0, out->est_candidates_per_step));
+        const double wcap = std::min(qcap, std::max(4194304.0, 4.0 * nn));
+        out->fixed_bytes = 48.0 * nn + (8.0 * kNCol + 1.0 + 4.0) * nn + 12.0 * qcap + 24.0 * wcap;
+        // a_gh + a_l of one step's grid, in the structure the auto cell edge selects for the
+        // a-priori density: chained heads (4 B x next_pow2(4n)) in ball mode, the open map
+        // (16 B x next_pow2(2n) slots + next_pow2(32n)-bit occupancy) in half-shell mode, plus the
+        // 32-byte entries {x, y, z, next}
+        const double m = choose_cell_factor(std::max(1.0, out->est_candidates_per_step) / std::max(1.0, nn));
+        const double n_u = std::max(1.0, nn);
+        const double chained = 4.0 * (double)next_pow2((uint64_t)(4.0 * n_u));
+        const double open = 16.0 * (double)next_pow2((uint64_t)(2.0 * n_u)) +
+                            (double)next_pow2((uint64_t)(32.0 * n_u)) / 8.0;
+        out->bytes_per_grid = (m < 2.0 ? open : chained) + 32.0 * nn;
+        out->grids_in_memory = std::max(0.0, ((double)mem_bytes - out->fixed_bytes) / out->bytes_per_grid);
+        out->rounds = out->grids_in_memory > 0.0 ? out->samples / out->grids_in_memory : INFINITY;
+        out->cell_factor = m;
+        return CD_OK;
+    } catch (...) {
+        return fail(CD_EINTERNAL, "unexpected C++ exception");
+    }
 }
 
 void cd_candidates_free(cd_candidate* c) { free(c); }

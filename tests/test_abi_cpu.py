@@ -83,3 +83,34 @@ def test_product_never_imports_oracle():
         txt = p.read_text()
         assert "import oracle" not in txt and "from oracle" not in txt, p
         assert "cd_oracle" not in txt and "liborc" not in txt, p
+
+
+def test_plan_extra_p_models(cds):
+    """cd_plan against PAPER.md Section IV-B as printed: Eq. 3 / Eq. 4, the
+    capacity rule c = max(c', 10^4) * 2 * 2 and g_ch = 16 c, o = t / s_ps
+    (with both window ends included, R4), p and r_c = o / p."""
+    n, d = 64000, 2.0
+    g = cds.plan(n, 0.0, 86400.0, 1.0, d, "grid", mem_bytes=24 << 30)
+    # Eq. 3 with s = 1 s, t = 86400 s, d = 2 km: 2.32e-9 * 64000^2 * 86400 * 2^1.75
+    assert g["est_candidates"] == pytest.approx(2.32e-9 * 4.096e9 * 86400.0 * 2.0 ** 1.75, rel=1e-12)
+    assert g["samples"] == 86401
+    assert g["capacity"] == pytest.approx(4 * g["est_candidates"], rel=1e-12)
+    assert g["capacity_bytes"] == pytest.approx(16 * g["capacity"], rel=1e-12)
+    assert g["est_candidates_per_step"] == pytest.approx(g["est_candidates"] / 86400.0, rel=1e-12)
+    h = cds.plan(n, 0.0, 86400.0, 9.0, d, "hybrid", mem_bytes=24 << 30)
+    # Eq. 4: 2.14e-9 n^2 s^(5/3) t d with s = 9 s
+    assert h["est_candidates"] == pytest.approx(2.14e-9 * 4.096e9 * 9.0 ** (5 / 3) * 86400.0 * 2.0, rel=1e-12)
+    assert h["samples"] == 9601
+    # the 10^4 floor of P:272 for a tiny screen
+    tiny = cds.plan(100, 0.0, 60.0, 1.0, 1.0, "grid", mem_bytes=1 << 30)
+    assert tiny["est_candidates"] < 1e4 and tiny["capacity"] == 4e4
+    # p and r_c as defined (P:239, P:251); p grows linearly with the free memory
+    for m in (8 << 30, 24 << 30, 180 << 30):
+        q = cds.plan(n, 0.0, 86400.0, 1.0, d, "grid", mem_bytes=m)
+        assert q["grids_in_memory"] == pytest.approx((m - q["fixed_bytes"]) / q["bytes_per_grid"], rel=1e-12)
+        assert q["rounds"] == pytest.approx(q["samples"] / q["grids_in_memory"], rel=1e-12)
+    # n^2 scaling of both models (the paper's "mainly the product of n, t and d")
+    g2 = cds.plan(2 * n, 0.0, 86400.0, 1.0, d, "grid", mem_bytes=24 << 30)
+    assert g2["est_candidates"] == pytest.approx(4 * g["est_candidates"], rel=1e-12)
+    with pytest.raises(cds.CdError):
+        cds.plan(n, 10.0, 0.0, 1.0, d, "grid", mem_bytes=1 << 30)
