@@ -68,9 +68,13 @@ static void hy_make(const orc_elements* el, int64_t i, hy_orbit* o)
     o->M0 = E0 - e * sin(E0);
 }
 
-/* mean anomaly of true anomaly f (forward Kepler relation, no solve), in (-pi, pi] */
+/* mean anomaly of true anomaly f (forward Kepler relation, no solve), in [-pi, pi]: f is first
+ * reduced to [-pi, pi], so that f/2 lies in [-pi/2, pi/2] and the half-angle formula returns the
+ * principal E (an unreduced f beyond pi would land E -- and M -- on another branch, 2 pi or 4 pi
+ * away, and a window whose ends fall on different branches would come out empty) */
 static double hy_mean_of_true(double f, double e)
 {
+    f = remainder(f, HY_TWO_PI);
     double E = 2.0 * atan2(sqrt(1.0 - e) * sin(0.5 * f), sqrt(1.0 + e) * cos(0.5 * f));
     return E - e * sin(E);
 }

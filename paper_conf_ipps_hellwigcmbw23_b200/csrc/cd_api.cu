@@ -651,7 +651,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     // are redone.  The candidate hook (Want::Cand) copies each accepted round's queue out, so it
     // runs unpipelined.
     const int depth = want == Want::Cand ? 1 : 2;
-    struct Round { int64_t k, Rk; int slot; size_t qcap; };   // qcap: the capacity it ran with
+    struct Round { int64_t k, Rk; int slot; size_t qcap, wcap, ocap; };   // capacities it ran with
     Round inflight[2];
     int nin = 0, next_slot = 0;
     auto enqueue_round = [&](int64_t kr, int64_t Rk, int slot) -> cd_status {
@@ -732,7 +732,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             const int slot = next_slot;
             next_slot ^= 1;
             TRY(enqueue_round(k, Rk, slot));
-            inflight[nin++] = Round{k, Rk, slot, qcap};
+            inflight[nin++] = Round{k, Rk, slot, qcap, wcap, ocap};
             k += Rk;
             continue;
         }
@@ -765,12 +765,12 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                 }
             }
             redo = true;
-        } else if (want == Want::Conj && hnwork > wcap) {
+        } else if (want == Want::Conj && hnwork > rd.wcap) {
             ++stats.retries;
-            wcap = (size_t)(hnwork * 1.25) + 1024;
+            wcap = std::max(wcap, (size_t)(hnwork * 1.25) + 1024);
             CU(w.alloc(wcap));
             redo = true;
-        } else if (want == Want::Conj && hctrl->n_conj > ocap) {
+        } else if (want == Want::Conj && hctrl->n_conj > rd.ocap) {
             ++stats.retries;
             const size_t ncap = std::max<size_t>(2 * ocap, (size_t)(hctrl->n_conj * 1.25) + 1024);
             DBuf<Conj> nb(st);
@@ -827,6 +827,23 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         hyb_before[1] = hctrl->n_coplanar;
         hyb_before[2] = hctrl->n_path;
         hyb_before[3] = hctrl->n_time;
+        // grow the work and output buffers ahead of need (a round that overflows is redone).
+        // Both reallocations are stream-ordered behind the round still in flight: the output
+        // copy moves the whole old buffer, including what that round appends; it is checked
+        // against the capacities it ran with (Round).
+        if (want == Want::Conj && hnwork > wcap / 2) {
+            wcap = std::max<size_t>(2 * wcap, 2 * hnwork);
+            CU(w.alloc(wcap));
+        }
+        if (want == Want::Conj && conj_before > ocap / 2) {
+            const size_t ncap = std::max<size_t>(2 * ocap, 4 * (size_t)conj_before);
+            DBuf<Conj> nb(st);
+            CU(nb.alloc(ncap));
+            CU(cudaMemcpyAsync(nb.p, R.conj.p, sizeof(Conj) * ocap, cudaMemcpyDeviceToDevice, st));
+            std::swap(R.conj.p, nb.p);
+            std::swap(R.conj.n, nb.n);
+            ocap = ncap;
+        }
         if (!settled) {   // first round done: pick the cell edge from the measured density
             const double m = choose_cell_factor((double)hctrl->n_cand / ((double)rd.Rk * (double)n));
             L = gc * m;

@@ -16,6 +16,9 @@
 // Surviving intervals become Brent work items (k_brent, shared with the grid variant); because
 // every filter is conservative the result is the set of minima below d owned by coarse steps.
 #include "cd_hybrid.h"
+#ifdef CD_DEBUG_FILTER
+#include <cstdio>
+#endif
 #include "cd_refine.cuh"
 
 using namespace cdk;
@@ -56,8 +59,11 @@ __device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o)
     o.pad = 0.0;
 }
 
+// mean anomaly of true anomaly f, in [-pi, pi]: f is reduced to [-pi, pi] first so the half-angle
+// formula stays on its principal branch (window ends on different branches would cancel a window)
 __device__ __forceinline__ double mean_of_true(double f, double e)
 {
+    f = remainder(f, kTwoPiH);
     double sf, cf;
     sincos(0.5 * f, &sf, &cf);
     const double E = 2.0 * atan2(sqrt(1.0 - e) * sf, sqrt(1.0 + e) * cf);
@@ -196,6 +202,10 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
                     }
                 }
         }
+#ifdef CD_DEBUG_FILTER
+        printf("filter i=%u j=%u k=%u sD=%.17g sA=%.17g sB=%.17g fA=%.17g fB=%.17g lo=%g hi=%g any=%d nwin=%d A.M0=%.17g A.nm=%.17g B.M0=%.17g B.nm=%.17g\n",
+               cd.i, cd.j, cd.step, sD, sA, sB, fA, fB, lo, hi, (int)any_node, nwin, A.M0, A.nm, B.M0, B.nm);
+#endif
         if (!any_node) count1(&ctrl->n_path);
         else if (nwin == 0) count1(&ctrl->n_time);
     }

@@ -99,3 +99,11 @@ def test_device_sort_merges_slices():
     got = cdist.records_to_numpy(t)
     exp = np.sort(rec, order=["i", "j", "step"], kind="stable")
     assert np.array_equal(got[["i", "j", "step"]], exp[["i", "j", "step"]])
+
+
+def test_hybrid_counter_rotating_wide_windows():
+    """Counter-rotating near-coplanar pairs: wide node windows whose true-anomaly ends straddle
+    f = 2 pi (the time filter's branch handling), GPU against the hybrid oracle."""
+    pop = popgen.counter_rotating(600, 7)
+    res, st = _check(pop, 0.0, 3600.0, 9.0, 5.0)
+    assert res["matched"] > 50

@@ -258,3 +258,22 @@ def test_full_size_sampled_steps(cfg4):
         Co = oracle.conjunctions(pop, t0, t1, dt, d, gc, Ko)
         Cs = Cg[Cg["step"] == k]
         parity.compare_conjunctions(pop, Cs, Co, t0, t1, dt, d, gc)
+
+
+@pytest.mark.gpu
+def test_config5_8m_sampled_steps():
+    """BASELINE config 5 (8,000,000 objects, the stress population): a few steps of the 7-day
+    window screened at full size, candidates and conjunctions compared with the oracle step by
+    step (the same launch configuration as any other call: auto cell edge, pipelined rounds)."""
+    pop, cfg = popgen.make_config(5)[:2]
+    d, dt = cfg.d, cfg.dt_grid
+    t0 = 3 * 86400.0 + 1234.0
+    t1 = t0 + 2 * dt
+    gc = oracle.cell_size(d, dt)
+    Kg = cds.candidates(pop, t0, t1, dt, d)
+    Cg = cds.screen(pop, t0, t1, dt, d)
+    Ko = oracle.candidates_grid(pop, t0, t1, dt, gc)
+    assert len(Ko) > 3 * 100000      # n^2 growth: ~64x the 1M population's rate per step
+    parity.compare_candidates(pop, Kg, Ko, t0, dt, gc)
+    Co = oracle.conjunctions(pop, t0, t1, dt, d, gc, Ko)
+    parity.compare_conjunctions(pop, Cg, Co, t0, t1, dt, d, gc)

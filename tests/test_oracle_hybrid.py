@@ -118,3 +118,21 @@ def test_hybrid_agrees_with_grid(orc):
         vrel = np.linalg.norm(v[0, 0] - v[0, 1])
         assert vrel > 15.6 * 0.999, (k, vrel)       # outside Eq. 1's speed assumption
     assert len(set(h) ^ set(g)) <= max(2, len(g) // 50)
+
+
+def test_conservative_counter_rotating_wide_windows(orc):
+    """Near-coplanar counter-rotating pairs (mutual inclination close to 180 deg): sin D is tiny,
+    the node windows are wide (|sin u| <= d / (q sin D) spans most of the orbit) and their
+    true-anomaly ends straddle f = 2 pi.  The filters must stay conservative there: the time
+    windows, converted through the mean anomaly, keep every minimum the unfiltered O3 finds."""
+    pop = popgen.counter_rotating(600, 7)
+    dt, d = 9.0, 5.0
+    gc = orc.cell_size(d, dt)
+    K = orc.candidates_grid(pop, 0.0, 3600.0, dt, gc)
+    full = orc.conjunctions(pop, 0.0, 3600.0, dt, d, gc, K)
+    hyb, counts = orc.hybrid(pop, 0.0, 3600.0, dt, d)
+    keep = (full["flags"] & orc.DEGENERATE) == 0
+    a = set(zip(full["i"][keep].tolist(), full["j"][keep].tolist(), full["step"][keep].tolist()))
+    b = set(zip(hyb["i"].tolist(), hyb["j"].tolist(), hyb["step"].tolist()))
+    assert len(a) > 50 and counts["coplanar"] < len(K)
+    assert a == b, (len(a - b), len(b - a))

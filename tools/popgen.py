@@ -339,3 +339,21 @@ def make_config(k: int, n: int | None = None):
 def random_population(n: int, seed: int, incl: str = "paper", shells: int = 0) -> dict:
     rng = np.random.default_rng(seed)
     return concat(walker_shells(rng, shells), base_mixture(rng, n - shells, incl))
+
+
+def counter_rotating(m: int, seed: int) -> dict:
+    """Near-coplanar counter-rotating population: one orbital plane flown both ways (mutual
+    inclinations within ~0.2 deg of 180 deg), a ~ 7000 +- 3 km, e < 4e-4, random omega and M.
+    Head-on encounters at ~15 km/s with very wide hybrid node windows (a stress case for the
+    time filter)."""
+    rng = np.random.default_rng(seed)
+    rows = []
+    for k in range(m):
+        inc, raan = 0.9, 0.4
+        if k % 2:
+            inc = math.pi - inc + rng.uniform(-2e-3, 2e-3)
+            raan = raan + math.pi + rng.uniform(-2e-3, 2e-3)
+        rows.append((7000.0 + rng.uniform(-3.0, 3.0), rng.uniform(0.0, 4e-4), inc, raan,
+                     rng.uniform(0, 2 * math.pi), rng.uniform(0, 2 * math.pi)))
+    arr = np.array(rows, dtype=np.float64)
+    return {k: np.ascontiguousarray(arr[:, c]) for c, k in enumerate(FIELDS)}
