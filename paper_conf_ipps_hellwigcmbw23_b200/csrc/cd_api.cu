@@ -21,6 +21,8 @@
 #include <string>
 #include <vector>
 
+#include <sys/mman.h>
+
 #include "../../include/cdscreen.h"
 #include "cd_internal.h"
 #include "cd_hybrid.h"
@@ -129,6 +131,111 @@ cd_status pinned_stage(Ctrl** out)
     return CD_OK;
 }
 
+// Per-host-thread page-locked bounce buffers for device -> pageable-host result copies: two
+// chunks, the DMA of one overlapping the host memcpy of the other (a direct copy into pageable
+// memory runs at a fraction of the link rate)
+constexpr size_t kBounceBytes = size_t(16) << 20;
+struct Bounce {
+    unsigned char* p = nullptr;
+    cudaEvent_t ev[2] = {nullptr, nullptr};
+    ~Bounce()
+    {
+        if (p) cudaFreeHost(p);
+        for (auto e : ev) if (e) cudaEventDestroy(e);
+    }
+};
+thread_local Bounce g_bounce;
+
+cudaError_t copy_to_pageable(void* dst, const void* src, size_t bytes, cudaStream_t st)
+{
+    if (bytes <= kBounceBytes / 4) {   // small: one direct copy
+        cudaError_t e = cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, st);
+        return e != cudaSuccess ? e : cudaStreamSynchronize(st);
+    }
+    if (!g_bounce.p) {
+        cudaError_t e = cudaMallocHost((void**)&g_bounce.p, 2 * kBounceBytes);
+        if (e != cudaSuccess) {
+            g_bounce.p = nullptr;
+            return e;
+        }
+        for (auto& ev : g_bounce.ev) {
+            e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+            if (e != cudaSuccess) return e;
+        }
+    }
+    const size_t nch = (bytes + kBounceBytes - 1) / kBounceBytes;
+    auto issue = [&](size_t c) -> cudaError_t {
+        const size_t off = c * kBounceBytes, len = std::min(kBounceBytes, bytes - off);
+        cudaError_t e = cudaMemcpyAsync(g_bounce.p + (c & 1) * kBounceBytes,
+                                        static_cast<const unsigned char*>(src) + off, len,
+                                        cudaMemcpyDeviceToHost, st);
+        return e != cudaSuccess ? e : cudaEventRecord(g_bounce.ev[c & 1], st);
+    };
+    cudaError_t e = issue(0);
+    for (size_t c = 0; c < nch && e == cudaSuccess; ++c) {
+        if (c + 1 < nch) e = issue(c + 1);
+        if (e != cudaSuccess) break;
+        e = cudaEventSynchronize(g_bounce.ev[c & 1]);
+        const size_t off = c * kBounceBytes, len = std::min(kBounceBytes, bytes - off);
+        memcpy(static_cast<unsigned char*>(dst) + off, g_bounce.p + (c & 1) * kBounceBytes, len);
+    }
+    return e;
+}
+
+// Per-device cache of the (unsorted) conjunction accumulation buffer (cudaMalloc'd): grow-only, handed from
+// call to call so a repeated or long screen does not regrow it (growing a stream-ordered pool by
+// hundreds of MB is a blocking driver call that stalls the round pipeline for up to ~1 s).  The
+// event orders the next user after the last use (the finalize sort) on the previous call's stream.
+struct ConjCache {
+    std::mutex mu;
+    Conj* p = nullptr;
+    size_t cap = 0;
+    cudaEvent_t ready = nullptr;
+};
+ConjCache g_conj_cache[64];
+
+// Take the cached buffer of device dev (waits on `st` for its last use); false if none / busy.
+bool conj_cache_take(int dev, cudaStream_t st, Conj** p, size_t* cap)
+{
+    if (dev < 0 || dev >= 64) return false;
+    ConjCache& c = g_conj_cache[dev];
+    std::lock_guard<std::mutex> lk(c.mu);
+    if (!c.p) return false;
+    if (c.ready) cudaStreamWaitEvent(st, c.ready, 0);
+    *p = c.p;
+    *cap = c.cap;
+    c.p = nullptr;
+    c.cap = 0;
+    return true;
+}
+
+// Return a buffer (its last use already enqueued on `st`); keeps the larger of cached / returned.
+void conj_cache_give(int dev, cudaStream_t st, Conj* p, size_t cap)
+{
+    if (!p) return;
+    if (dev < 0 || dev >= 64) {
+        cudaFree(p);
+        return;
+    }
+    ConjCache& c = g_conj_cache[dev];
+    std::lock_guard<std::mutex> lk(c.mu);
+    if (c.p && c.cap >= cap) {
+        cudaFree(p);
+        return;
+    }
+    if (c.p) cudaFree(c.p);   // (cudaFree synchronises the device: its last use is done)
+    if (!c.ready && cudaEventCreateWithFlags(&c.ready, cudaEventDisableTiming) != cudaSuccess) {
+        c.ready = nullptr;
+        cudaFree(p);
+        c.p = nullptr;
+        c.cap = 0;
+        return;
+    }
+    cudaEventRecord(c.ready, st);
+    c.p = p;
+    c.cap = cap;
+}
+
 // Compute capability per device, queried once (cudaGetDeviceProperties costs milliseconds).
 int g_cc[64];   // 0 = not yet queried, else major * 10 + minor
 
@@ -148,6 +255,7 @@ struct Owner {
     bool device;
     void* p;
     cudaStream_t st;   // device results: released stream-ordered on the call's stream
+    size_t host_bytes; // host results: size of the anonymous mapping (munmap)
 };
 
 // Optional per-phase device timing (cd_options.profile_phases): CUDA events recorded on the
@@ -472,11 +580,80 @@ size_t initial_qcap(int64_t n, double est_step)
     return qcap;
 }
 
+// The conjunction accumulation buffer: plain cudaMalloc (a few ms even for GBs, where growing the
+// stream-ordered pool mid-screen was measured at up to ~1 s of blocked host thread), grow-only;
+// a replaced buffer is retired and freed after the call's final synchronisation.
+struct ConjBuf {
+    Conj* p = nullptr;
+    size_t n = 0;
+    std::vector<Conj*> retired;
+    ConjBuf() = default;
+    ConjBuf(const ConjBuf&) = delete;
+    ConjBuf& operator=(const ConjBuf&) = delete;
+    ~ConjBuf()
+    {
+        for (Conj* r : retired) cudaFree(r);
+        if (p) cudaFree(p);
+    }
+    // new buffer of `count` records; the first `keep` records are copied over (stream-ordered)
+    cudaError_t grow(size_t count, size_t keep, cudaStream_t st)
+    {
+        Conj* np = nullptr;
+        cudaError_t e = cudaMalloc((void**)&np, sizeof(Conj) * (count ? count : 1));
+        if (e != cudaSuccess) return e;
+        if (p && keep) e = cudaMemcpyAsync(np, p, sizeof(Conj) * keep, cudaMemcpyDeviceToDevice, st);
+        if (p) retired.push_back(p);
+        p = np;
+        n = count;
+        return e;
+    }
+    Conj* detach()
+    {
+        Conj* q = p;
+        p = nullptr;
+        n = 0;
+        return q;
+    }
+};
+
 struct Result {
-    DBuf<Conj> conj;        // unsorted conjunction records (internal ids)
+    ConjBuf conj;           // unsorted conjunction records (internal ids)
     size_t n_conj = 0;
     DBuf<Cand> cand;        // accumulated candidates (cd_candidates)
     size_t n_cand = 0;
+    // host result buffer (outputs on the host): an anonymous mapping advised for transparent
+    // huge pages, so the copy-out faults in 2 MB pages instead of 4 KB ones (a 350 MB result
+    // otherwise spends hundreds of ms in page faults); released with munmap
+    void* host = nullptr;
+    size_t host_bytes = 0;
+    ~Result() { release_host(host, host_bytes); }
+    static void release_host(void* p, size_t bytes)
+    {
+        if (p) munmap(p, bytes);
+    }
+    bool alloc_host(size_t count)
+    {
+        release_host(host, host_bytes);
+        host = nullptr;
+        const size_t huge = size_t(2) << 20;
+        host_bytes = ((sizeof(Conj) * count + huge - 1) / huge) * huge;
+        void* p = mmap(nullptr, host_bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+        if (p == MAP_FAILED) {
+            host_bytes = 0;
+            return false;
+        }
+        madvise(p, host_bytes, MADV_HUGEPAGE);   // best effort
+        host = p;
+        return true;
+    }
+    void* take_host(size_t* bytes)
+    {
+        void* p = host;
+        *bytes = host_bytes;
+        host = nullptr;
+        host_bytes = 0;
+        return p;
+    }
 };
 
 // The screening loop over this rank's step slice.
@@ -510,7 +687,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     g.max_walk = (uint32_t)std::min<int64_t>(n + 1, 0xfffffffe);
     RefineParams P{t0, t1, dt, d, gc, nullptr};
 
-    R.conj.st = R.cand.st = st;
+    R.cand.st = st;
     if (ke <= kb || n < 2) return CD_OK;
 
     const uint64_t M = next_pow2((uint64_t)std::max<int64_t>(2 * n, 64));   // >= 2n slots (power of 2)
@@ -598,7 +775,18 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     DBuf<Work> w(st);
     if (want == Want::Conj) CU(w.alloc(wcap));
     size_t ocap = size_t(1) << 20;
-    if (want == Want::Conj) CU(R.conj.alloc(ocap));
+    if (want == Want::Conj) {
+        Conj* cp = nullptr;
+        size_t cc = 0;
+        if (conj_cache_take(C.dev, st, &cp, &cc) && cc >= ocap) {
+            R.conj.p = cp;
+            R.conj.n = cc;
+            ocap = cc;
+        } else {
+            if (cp) cudaFree(cp);
+            CU(R.conj.grow(ocap, 0, st));
+        }
+    }
     size_t ccap = want == Want::Cand ? (size_t(1) << 20) : 0;
     if (want == Want::Cand) CU(R.cand.alloc(ccap));
 
@@ -773,12 +961,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         } else if (want == Want::Conj && hctrl->n_conj > rd.ocap) {
             ++stats.retries;
             const size_t ncap = std::max<size_t>(2 * ocap, (size_t)(hctrl->n_conj * 1.25) + 1024);
-            DBuf<Conj> nb(st);
-            CU(nb.alloc(ncap));
-            if (conj_before)
-                CU(cudaMemcpyAsync(nb.p, R.conj.p, sizeof(Conj) * conj_before, cudaMemcpyDeviceToDevice, st));
-            std::swap(R.conj.p, nb.p);
-            std::swap(R.conj.n, nb.n);
+            CU(R.conj.grow(ncap, conj_before, st));
             ocap = ncap;
             redo = true;
         }
@@ -835,13 +1018,15 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             wcap = std::max<size_t>(2 * wcap, 2 * hnwork);
             CU(w.alloc(wcap));
         }
-        if (want == Want::Conj && conj_before > ocap / 2) {
-            const size_t ncap = std::max<size_t>(2 * ocap, 4 * (size_t)conj_before);
-            DBuf<Conj> nb(st);
-            CU(nb.alloc(ncap));
-            CU(cudaMemcpyAsync(nb.p, R.conj.p, sizeof(Conj) * ocap, cudaMemcpyDeviceToDevice, st));
-            std::swap(R.conj.p, nb.p);
-            std::swap(R.conj.n, nb.n);
+        // output: grown once the projected total (x 1.25) would not fit, to 1.5x the projection,
+        // so a long screen grows it early (little to copy) and rarely
+        const double done_steps = (double)(rd.k + rd.Rk - kb);
+        const double proj_conj = (double)conj_before * (double)(ke - kb) / std::max(1.0, done_steps);
+        if (want == Want::Conj && settled && (1.25 * proj_conj > (double)ocap || conj_before > ocap * 9 / 10)) {
+            const size_t ncap = std::max<size_t>(2 * ocap, (size_t)(1.5 * proj_conj));
+            DBG("grow: output", (long long)ocap, (long long)ncap);
+            CU(R.conj.grow(ncap, ocap, st));
+            DBG("grow: allocated");
             ocap = ncap;
         }
         if (!settled) {   // first round done: pick the cell edge from the measured density
@@ -915,19 +1100,30 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
             CU(finalize_conj(R.conj.p, R.n_conj, S.perm.p, sorted.p, C.st, C.lc));
             C.pt.stop();
         }
+        // the accumulation buffer goes back to the per-device cache (its last use, the sort,
+        // is enqueued on C.st)
+        const size_t cap = R.conj.n;
+        conj_cache_give(C.dev, C.st, R.conj.detach(), cap);
     }
-    Owner* own = new Owner{o.outputs_on_device != 0, nullptr, C.own_stream ? nullptr : C.st};
+    Owner* own = new Owner{o.outputs_on_device != 0, nullptr, C.own_stream ? nullptr : C.st, 0};
     if (R.n_conj) {
         if (o.outputs_on_device) {
             own->p = sorted.detach();
         } else {
-            void* h = malloc(sizeof(cd_conjunction) * R.n_conj);
+            size_t hb = 0;
+            void* h = R.alloc_host(R.n_conj) ? R.take_host(&hb) : nullptr;
             if (!h) {
                 delete own;
                 return fail(CD_ENOMEM, "host allocation of %zu records failed", R.n_conj);
             }
-            CU(cudaMemcpyAsync(h, sorted.p, sizeof(cd_conjunction) * R.n_conj, cudaMemcpyDeviceToHost, C.st));
             own->p = h;
+            own->host_bytes = hb;
+            const cudaError_t e = copy_to_pageable(h, sorted.p, sizeof(cd_conjunction) * R.n_conj, C.st);
+            if (e != cudaSuccess) {
+                Result::release_host(h, hb);
+                delete own;
+                return fail(CD_ECUDA, "copy-out: %s", cudaGetErrorString(e));
+            }
         }
     }
     DBG("screen: finalized");
@@ -1093,7 +1289,7 @@ void cd_conjunctions_free(cd_conjunctions* c)
             // caller queued on the call's stream (the legacy default stream if the library
             // created its own)
             if (own->device) cudaFreeAsync(own->p, own->st);
-            else free(own->p);
+            else munmap(own->p, own->host_bytes);
         }
         delete own;
     }
