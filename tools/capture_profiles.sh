@@ -1,12 +1,15 @@
 #!/bin/bash
-# GPU-box capture for profiles/: launch list of one bench-shaped call and one ncu --set full
-# capture of the dominant kernel.  Output under gpurun_out/$1/.
+# GPU-box capture for profiles/: launch list of the bench command (cold-cache, serialised:
+# compare shares, not absolutes), ncu --set full of the dominant kernel (grid k_step, steady
+# state) and of the hybrid variant's kernels.  Output under gpurun_out/$1/.
 set -e
 OUT=gpurun_out/${1:-prof}
 mkdir -p $OUT
-# launch list (cold-cache, serialised: compare shares, not absolutes)
-ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
-    python tools/profile_step.py --steps 200 > $OUT/launches.log 2>&1 || true
-# full section set of the fused step kernel (steady state launches)
-ncu --set full --clock-control none --import-source on -k regex:k_step -s 20 -c 3 \
-    -o $OUT/k_step python tools/profile_step.py --steps 40 > $OUT/full.log 2>&1 || true
+ncu --metrics gpu__time_duration.sum --clock-control none -c 3000 --csv --log-file $OUT/launches.csv \
+    python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-hybrid --e2e-steps 0 --no-profile > $OUT/launches.log 2>&1 || true
+ncu --set full --clock-control none --import-source on -k regex:k_step -s 60 -c 3 \
+    -o $OUT/k_step python tools/profile_step.py --steps 400 > $OUT/full.log 2>&1 || true
+ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/hyb_launches.csv \
+    python tools/profile_step.py --variant hybrid --steps 200 > $OUT/hyb_launches.log 2>&1 || true
+ncu --set full --clock-control none --import-source on -k regex:"k_step|k_hybrid_filter" -s 30 -c 4 \
+    -o $OUT/hyb python tools/profile_step.py --variant hybrid --steps 200 > $OUT/hyb_full.log 2>&1 || true
