@@ -43,8 +43,12 @@ def build(force: bool = False) -> Path:
     return LIB
 
 
+PROPAGATORS = {"kepler": 0, "j2": 1}
+
+
 class _Elements(C.Structure):
-    _fields_ = [(k, C.POINTER(C.c_double)) for k in ("a", "e", "inc", "raan", "argp", "nu0")]
+    _fields_ = [(k, C.POINTER(C.c_double)) for k in ("a", "e", "inc", "raan", "argp", "nu0")] + \
+        [("model", C.c_int)]
 
 
 _lib = None
@@ -57,6 +61,8 @@ def lib():
         L = C.CDLL(str(LIB))
         P = C.POINTER
         L.orc_mu.restype = C.c_double
+        L.orc_j2.restype = C.c_double
+        L.orc_earth_radius.restype = C.c_double
         L.orc_num_threads.restype = C.c_int
         L.orc_kepler_newton.restype = C.c_double
         L.orc_kepler_newton.argtypes = [C.c_double, C.c_double]
@@ -116,7 +122,9 @@ class _Pop:
     def __init__(self, pop):
         self.arrs = [_f64(pop[k]) for k in ("a", "e", "inc", "raan", "argp", "nu0")]
         self.n = int(self.arrs[0].shape[0])
-        self.s = _Elements(*[_dp(a) for a in self.arrs])
+        # the force model travels with the population: pop["propagator"] in PROPAGATORS
+        self.model = PROPAGATORS[pop.get("propagator", "kepler")] if hasattr(pop, "get") else 0
+        self.s = _Elements(*[_dp(a) for a in self.arrs], self.model)
 
     @property
     def ref(self):
@@ -125,6 +133,20 @@ class _Pop:
 
 def mu() -> float:
     return lib().orc_mu()
+
+
+def j2() -> float:
+    return lib().orc_j2()
+
+
+def earth_radius() -> float:
+    return lib().orc_earth_radius()
+
+
+def with_propagator(pop, name):
+    """The population with its force model set ("kepler" or "j2")."""
+    assert name in PROPAGATORS, name
+    return dict(pop, propagator=name)
 
 
 def num_threads() -> int:
@@ -209,6 +231,8 @@ def pair_distance(pop, i, j, times):
 def pair_filter(pop, i, j, d, tlo, thi):
     """Hybrid filter chain for one pair over [tlo, thi]: (flags, [(lo, hi), ...])."""
     P = _Pop(pop)
+    if P.model:
+        raise ValueError("hybrid filters assume fixed orbit planes: Kepler propagator only")
     iv = np.zeros(64)
     niv = C.c_int()
     f = lib().orc_pair_filter(P.ref, int(i), int(j), float(d), float(tlo), float(thi), _dp(iv), 32,
@@ -220,6 +244,8 @@ def hybrid(pop, t0, t1, dt, d, v_margin=7.8, k_begin=0, k_end=-1):
     """Hybrid variant end to end (O4): conjunctions and the filter-stage counts
     (candidates, ap_rejected, coplanar, path_rejected, time_rejected, time_window_work)."""
     P = _Pop(pop)
+    if P.model:
+        raise ValueError("hybrid filters assume fixed orbit planes: Kepler propagator only")
     gc = cell_size(d, dt, v_margin)
     out = C.c_void_p()
     counts = (C.c_int64 * 6)()

@@ -12,6 +12,8 @@
  *
  * Levels:
  *   O1 propagate      -- two-body Kepler, Newton-Raphson on E - e sin E = M
+ *   O1' J2 secular    -- the same with secular J2 rates of Omega, omega, M ("other
+ *                        propagators"; Vallado [41] Section 9.6), orc_elements.model = 1
  *   O2 candidates     -- K = {(i,j,k): i<j, |r_i(t_k) - r_j(t_k)| < g_c}
  *                        brute force O(n^2) per step, and a plain sorted-cell grid with 27 neighbours
  *   O3 conjunctions   -- all local minima of D(t) = |r_i - r_j| inside the owner cell of step k
@@ -61,7 +63,37 @@ double orc_kepler_newton(double M, double e)
 typedef struct {
     double a, e, b, nmean, M0;
     double P[3], Q[3];
+    /* J2 secular model (ORC_PROP_J2): elements at epoch and their secular rates */
+    int j2;
+    double inc, raan0, argp0, draan, dargp;
 } orc_orbit;
+
+/* ------------------------------------------------------------------------------------------
+ * O1': J2 secular propagator ("other propagators instead of the Kepler
+ * Contour solver").  First-order secular effect of Earth's oblateness J2 on the mean
+ * elements, Vallado & McClain [41] Section 9.6 (the paper's ref. [41]):
+ *     p = a (1 - e^2),  n0 = sqrt(mu / a^3),  k = J2 (R_E / p)^2
+ *     dM/dt     = n0 [1 + (3/2) k sqrt(1 - e^2) (1 - (3/2) sin^2 i)]
+ *     dOmega/dt = -(3/2) n0 k cos i
+ *     domega/dt =  (3/4) n0 k (4 - 5 sin^2 i)
+ * a, e, i constant; the position at t is the two-body position of the elements
+ * (a, e, i, Omega0 + dOmega/dt t, omega0 + domega/dt t, M0 + dM/dt t).  J2 and R_E: EGM-96 /
+ * WGS-84 values (reading R19).
+ * ------------------------------------------------------------------------------------------ */
+double orc_j2(void) { return 1.08262668e-3; }
+double orc_earth_radius(void) { return 6378.137; }
+
+static void orc_perifocal(double raan, double inc, double argp, double P[3], double Q[3])
+{
+    double cO = cos(raan), sO = sin(raan), cw = cos(argp), sw = sin(argp);
+    double ci = cos(inc), si = sin(inc);
+    P[0] = cO * cw - sO * sw * ci;
+    P[1] = sO * cw + cO * sw * ci;
+    P[2] = sw * si;
+    Q[0] = -cO * sw - sO * cw * ci;
+    Q[1] = -sO * sw + cO * cw * ci;
+    Q[2] = cw * si;
+}
 
 /* Per-object constants: perifocal unit vectors P, Q (Fig. 8: Omega, i, omega), mean motion,
  * mean anomaly at epoch from the true anomaly nu0 (P:166 element set; R#2). */
@@ -69,20 +101,28 @@ static void orc_make_orbit(const orc_elements* el, int64_t idx, orc_orbit* o)
 {
     double a = el->a[idx], e = el->e[idx], inc = el->inc[idx];
     double raan = el->raan[idx], argp = el->argp[idx], nu0 = el->nu0[idx];
-    double cO = cos(raan), sO = sin(raan), cw = cos(argp), sw = sin(argp);
-    double ci = cos(inc), si = sin(inc);
-    o->P[0] = cO * cw - sO * sw * ci;
-    o->P[1] = sO * cw + cO * sw * ci;
-    o->P[2] = sw * si;
-    o->Q[0] = -cO * sw - sO * cw * ci;
-    o->Q[1] = -sO * sw + cO * cw * ci;
-    o->Q[2] = cw * si;
+    orc_perifocal(raan, inc, argp, o->P, o->Q);
     o->a = a;
     o->e = e;
     o->b = a * sqrt(1.0 - e * e);
     o->nmean = sqrt(orc_mu() / (a * a * a));
     double E0 = 2.0 * atan2(sqrt(1.0 - e) * sin(0.5 * nu0), sqrt(1.0 + e) * cos(0.5 * nu0));
     o->M0 = E0 - e * sin(E0);
+    o->j2 = el->model == ORC_PROP_J2;
+    o->inc = inc;
+    o->raan0 = raan;
+    o->argp0 = argp;
+    o->draan = 0.0;
+    o->dargp = 0.0;
+    if (o->j2) {   /* Vallado [41] Section 9.6, see O1' above */
+        double p = a * (1.0 - e * e);
+        double k = orc_j2() * (orc_earth_radius() / p) * (orc_earth_radius() / p);
+        double n0 = o->nmean;
+        double s2 = sin(inc) * sin(inc);
+        o->nmean = n0 * (1.0 + 1.5 * k * sqrt(1.0 - e * e) * (1.0 - 1.5 * s2));
+        o->draan = -1.5 * n0 * k * cos(inc);
+        o->dargp = 0.75 * n0 * k * (4.0 - 5.0 * s2);
+    }
 }
 
 /* Position (and optionally velocity) at time t (seconds from epoch). */
@@ -95,14 +135,33 @@ static void orc_state(const orc_orbit* o, double t, double r[3], double v[3])
     double cE = cos(E), sE = sin(E);
     double x = o->a * (cE - o->e);
     double y = o->b * sE;
+    double P[3], Q[3];
+    if (o->j2) {   /* O1': the orbit plane and perigee at time t */
+        orc_perifocal(o->raan0 + o->draan * t, o->inc, o->argp0 + o->dargp * t, P, Q);
+    } else {
+        for (int c = 0; c < 3; ++c) {
+            P[c] = o->P[c];
+            Q[c] = o->Q[c];
+        }
+    }
     for (int c = 0; c < 3; ++c)
-        r[c] = x * o->P[c] + y * o->Q[c];
+        r[c] = x * P[c] + y * Q[c];
     if (v) {
-        double rr = o->a * (1.0 - o->e * cE);
-        double k = sqrt(orc_mu() * o->a) / rr;
-        double s1e2 = sqrt(1.0 - o->e * o->e);
+        /* dE/dt = n / (1 - e cos E) with n the mean-anomaly rate (n0, or the J2 dM/dt) */
+        double rr = 1.0 - o->e * cE;
+        double k = o->nmean / rr;
         for (int c = 0; c < 3; ++c)
-            v[c] = k * (-sE * o->P[c] + s1e2 * cE * o->Q[c]);
+            v[c] = k * (-o->a * sE * P[c] + o->b * cE * Q[c]);
+        if (o->j2) {
+            /* d/dt of the rotating plane: dOmega/dt z x r + domega/dt h x r, h = P x Q */
+            double h[3] = {P[1] * Q[2] - P[2] * Q[1], P[2] * Q[0] - P[0] * Q[2],
+                           P[0] * Q[1] - P[1] * Q[0]};
+            double hxr[3] = {h[1] * r[2] - h[2] * r[1], h[2] * r[0] - h[0] * r[2],
+                             h[0] * r[1] - h[1] * r[0]};
+            double zxr[3] = {-r[1], r[0], 0.0};
+            for (int c = 0; c < 3; ++c)
+                v[c] += o->draan * zxr[c] + o->dargp * hxr[c];
+        }
     }
 }
 

@@ -8,8 +8,11 @@
 extern "C" {
 #endif
 
+enum { ORC_PROP_KEPLER = 0, ORC_PROP_J2 = 1 };
+
 typedef struct {
     const double *a, *e, *inc, *raan, *argp, *nu0; /* km, -, rad, rad, rad, rad */
+    int model;                                     /* ORC_PROP_KEPLER or ORC_PROP_J2 */
 } orc_elements;
 
 typedef struct { uint32_t i, j, step; } orc_candidate;
@@ -24,6 +27,8 @@ typedef struct {
 } orc_conjunction;
 
 double  orc_mu(void);
+double  orc_j2(void);
+double  orc_earth_radius(void);
 int     orc_num_threads(void);
 double  orc_kepler_newton(double M, double e);
 int64_t orc_num_steps(double t0, double t1, double dt);

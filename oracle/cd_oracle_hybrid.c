@@ -170,6 +170,8 @@ static int hy_filter(const hy_orbit* A, const hy_orbit* B, double d, double tlo,
 int orc_pair_filter(const orc_elements* el, int64_t i, int64_t j, double d, double tlo, double thi,
                     double* iv, int cap, int* niv)
 {
+    if (el->model != ORC_PROP_KEPLER)   /* the filters assume fixed orbit planes (Kepler) */
+        return -1;
     hy_orbit A, B;
     hy_make(el, i, &A);
     hy_make(el, j, &B);
@@ -230,6 +232,10 @@ static int hy_cmp(const void* x, const void* y)
 int64_t orc_hybrid(const orc_elements* el, int64_t n, double t0, double t1, double dt, double d,
                    double gc, int64_t k_begin, int64_t k_end, void** out, int64_t* counts)
 {
+    if (el->model != ORC_PROP_KEPLER) {   /* the filters assume fixed orbit planes (Kepler) */
+        *out = NULL;
+        return -1;
+    }
     orc_candidate* cand = NULL;
     int64_t nc = orc_candidates_grid(el, n, t0, t1, dt, gc, 0.0, NULL, k_begin, k_end, &cand);
     /* plain serial-per-candidate evaluation, OpenMP over candidates */
