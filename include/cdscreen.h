@@ -42,7 +42,7 @@
 extern "C" {
 #endif
 
-#define CD_ABI_VERSION 1
+#define CD_ABI_VERSION 2   /* 2: cd_options.propagator */
 
 typedef enum {
     CD_OK = 0,
@@ -54,6 +54,19 @@ typedef enum {
     CD_EINTERNAL = 6, /* internal invariant violated                                           */
     CD_ENODEV = 7     /* no CUDA device / the library was not built for this device            */
 } cd_status;
+
+/* Propagator of the screen (two-body Kepler with the Contour solver [43]; P:333 names
+ * "other propagators instead of the Kepler Contour solver" as future work). */
+typedef enum {
+    CD_PROP_KEPLER = 0, /* two-body Kepler, Contour solver (the paper's propagator)                */
+    CD_PROP_J2 = 1      /* + first-order secular J2 drift of Omega, omega and M (Vallado &
+                           McClain [41] Sec. 9.6; J2 = 1.08262668e-3, R_E = 6378.137 km):
+                           dM/dt = n0 [1 + 1.5 k sqrt(1-e^2) (1 - 1.5 sin^2 i)],
+                           dOmega/dt = -1.5 n0 k cos i, domega/dt = 0.75 n0 k (4 - 5 sin^2 i),
+                           k = J2 (R_E / (a (1 - e^2)))^2, n0 = sqrt(mu/a^3); a, e, i constant.
+                           Grid variant and cd_propagate only (the hybrid filters assume fixed
+                           orbit planes: CD_HYBRID with CD_PROP_J2 is CD_EINVAL)                 */
+} cd_propagator;
 
 typedef enum {
     CD_GRID = 0,   /* grid-based variant                               */
@@ -138,6 +151,7 @@ typedef struct {
                                  2 = chained spatial hash (lists per hashed bucket, one atomic
                                  exchange per object); 0 = default (2).  Results are identical. */
     cd_stats* stats;          /* optional output                                              */
+    int propagator;           /* cd_propagator; default CD_PROP_KEPLER                        */
 } cd_options;
 
 /* Fill *opt with the defaults above. */

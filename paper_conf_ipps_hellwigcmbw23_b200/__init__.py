@@ -20,6 +20,8 @@ LIB_PATH = PKG / "libcdscreen.so"
 
 CD_OK, CD_EINVAL, CD_ENOMEM, CD_ECUDA, CD_ENCCL, CD_ERANGE, CD_EINTERNAL, CD_ENODEV = range(8)
 CD_GRID, CD_HYBRID = 0, 1
+CD_PROP_KEPLER, CD_PROP_J2 = 0, 1
+PROPAGATORS = {"kepler": CD_PROP_KEPLER, "j2": CD_PROP_J2}
 CD_FLAG_DEGENERATE = 2
 CD_FLAG_COPLANAR = 4
 FIELDS = ("a", "e", "inc", "raan", "argp", "nu0")
@@ -82,7 +84,7 @@ class cd_options(C.Structure):
                 ("kepler_points", C.c_int), ("cell_factor", C.c_double),
                 ("batch_object_steps", C.c_size_t), ("round_steps", C.c_size_t),
                 ("profile_phases", C.c_int), ("l2_persist", C.c_int), ("grid_table", C.c_int),
-                ("stats", C.POINTER(cd_stats))]
+                ("stats", C.POINTER(cd_stats)), ("propagator", C.c_int)]
 
 
 class cd_plan_info(C.Structure):
@@ -207,6 +209,8 @@ class _Elements:
     tensors -> device pointers (inputs_on_device)."""
 
     def __init__(self, pop):
+        # optional force model carried by the population dict ("kepler" / "j2")
+        self.propagator = pop.get("propagator") if hasattr(pop, "get") else None
         first = pop["a"]
         self.on_device = hasattr(first, "is_cuda") and bool(first.is_cuda)
         if self.on_device:
@@ -223,7 +227,7 @@ class _Elements:
 def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None, stream=None,
                  cell_factor=None, batch_object_steps=None, round_steps=None,
                  outputs_on_device=False, inputs_on_device=False, profile_phases=False,
-                 l2_persist=None, grid_table=None):
+                 l2_persist=None, grid_table=None, propagator=None):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -249,6 +253,8 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
         o.l2_persist = int(bool(l2_persist))
     if grid_table is not None:
         o.grid_table = int(grid_table)
+    if propagator is not None:
+        o.propagator = PROPAGATORS[propagator] if isinstance(propagator, str) else int(propagator)
     return o
 
 
@@ -272,6 +278,7 @@ def screen(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
     """Conjunctions as a structured numpy array (CONJ_DTYPE), sorted by (i, j, step)."""
     E = _Elements(pop)
     st = cd_stats()
+    kw.setdefault("propagator", E.propagator)
     opt = make_options(inputs_on_device=E.on_device, **kw)
     if opt.stream is None and E.on_device:
         opt.stream = _torch_stream()
@@ -295,6 +302,7 @@ def candidates(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
     """The level-1 candidate set K as a structured numpy array (CAND_DTYPE), sorted."""
     E = _Elements(pop)
     st = cd_stats()
+    kw.setdefault("propagator", E.propagator)
     opt = make_options(inputs_on_device=E.on_device, **kw)
     opt.stats = C.pointer(st)
     p = C.c_void_p()
@@ -318,6 +326,7 @@ def propagate(pop, times, velocity=False, **kw):
     t = np.ascontiguousarray(np.atleast_1d(np.asarray(times, dtype=np.float64)))
     xyz = np.zeros((t.size, E.n, 3))
     v = np.zeros((t.size, E.n, 3)) if velocity else None
+    kw.setdefault("propagator", E.propagator)
     opt = make_options(inputs_on_device=E.on_device, **kw)
     _check(cd_propagate(E.s, E.n, t.ctypes.data, t.size, xyz.ctypes.data,
                         v.ctypes.data if velocity else None, opt))

@@ -428,6 +428,8 @@ cd_status validate_scalars(size_t n, double t0, double t1, double dt, double d, 
         return fail(CD_EINVAL, "need cell_factor = 0 (auto) or >= 1");
     if (o.n_ranks < 1 || o.rank < 0 || o.rank >= o.n_ranks)
         return fail(CD_EINVAL, "need 0 <= rank < n_ranks");
+    if (o.propagator != CD_PROP_KEPLER && o.propagator != CD_PROP_J2)
+        return fail(CD_EINVAL, "unknown propagator %d", o.propagator);
     for (int c = 0; c < 3; ++c)
         if (!is_fin(o.grid_origin[c])) return fail(CD_EINVAL, "grid_origin must be finite");
     const double kk = std::floor((t1 - t0) / dt) + 1.0;
@@ -465,6 +467,7 @@ struct OrbitSet {
     DBuf<uint8_t> cls;
     DBuf<uint32_t> perm;   // internal -> caller index
     int64_t n0 = 0;        // class-0 objects (sorted first)
+    int j2 = 0;            // CD_PROP_J2 records
     Orbits view() const
     {
         Orbits O;
@@ -472,6 +475,7 @@ struct OrbitSet {
         O.cls = cls.p;
         O.n = (int64_t)perm.n;
         O.n0 = n0;
+        O.j2 = j2;
         return O;
     }
 };
@@ -518,9 +522,10 @@ cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_opti
     unsigned long long hn0 = 0;
     CU(cudaMemcpyAsync(&hn0, n0.p, sizeof hn0, cudaMemcpyDeviceToHost, st));
     CU(sort_pairs_u32(key.p, keyo.p, idx.p, S.perm.p, n, 3, st, C.lc));
-    CU(S.rec.alloc((size_t)kNCol * n));
+    S.j2 = o.propagator == CD_PROP_J2;
+    CU(S.rec.alloc((size_t)(S.j2 ? kNCol : kDOm) * n));   // the J2 columns only when used
     CU(S.cls.alloc(n));
-    CU(launch_build_records(E, S.perm.p, (int64_t)n, S.rec.p, S.cls.p, st, C.lc));
+    CU(launch_build_records(E, S.perm.p, (int64_t)n, S.rec.p, S.cls.p, S.j2, st, C.lc));
     C.pt.stop();
     CU(cudaStreamSynchronize(st));   // hn0 is needed on the host
     S.n0 = (int64_t)hn0;
@@ -1075,6 +1080,8 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
     out->_owner = nullptr;
     const cd_options o = opt ? *opt : defaults();
     if (mode != CD_GRID && mode != CD_HYBRID) return fail(CD_EINVAL, "unknown mode %d", (int)mode);
+    if (mode == CD_HYBRID && o.propagator != CD_PROP_KEPLER)
+        return fail(CD_EINVAL, "CD_HYBRID needs CD_PROP_KEPLER (the filters assume fixed orbit planes)");
     int64_t K = 0;
     TRY(validate_scalars(n, t0, t1, dt, d, o, &K));
     cd_stats stats;
@@ -1159,6 +1166,7 @@ void cd_options_init(cd_options* o)
     o->cell_factor = 0.0;   // auto (1.0 = the paper's cell edge g_c, 27-cell neighbourhood)
     o->l2_persist = 0;
     o->grid_table = 0;
+    o->propagator = CD_PROP_KEPLER;
 }
 
 cd_status cd_screen(const cd_elements* el, size_t n, double t0, double t1, double dt, double d,
@@ -1328,7 +1336,7 @@ cd_status cd_plan(size_t n, double t0, double t1, double dt, double d, cd_mode m
         // permutation, a_ch the round's candidate queue (12 B) and work items (24 B)
         const double qcap = (double)initial_qcap((int64_t)n, std::max(1.0, out->est_candidates_per_step));
         const double wcap = std::min(qcap, std::max(4194304.0, 4.0 * nn));
-        out->fixed_bytes = 48.0 * nn + (8.0 * kNCol + 1.0 + 4.0) * nn + 12.0 * qcap + 24.0 * wcap;
+        out->fixed_bytes = 48.0 * nn + (8.0 * kDOm + 1.0 + 4.0) * nn + 12.0 * qcap + 24.0 * wcap;
         // a_gh + a_l of one step's grid, in the structure the auto cell edge selects for the
         // a-priori density: chained heads (4 B x next_pow2(4n)) in ball mode, the open map
         // (16 B x next_pow2(2n) slots + next_pow2(32n)-bit occupancy) in half-shell mode, plus the

@@ -27,8 +27,16 @@ enum Col : int {
     kEcr = 10, kEsr = 11,            // e cos(rho), e sin(rho), rho = e/2   (real nodes)
     kTab = 12,                       // 4 per symmetric interior pair: e cos(rho c_j),
                                      // e sin(rho c_j), cosh(rho s_j), sinh(rho s_j)
-    kNCol = 12 + 28
+    // J2 secular propagator (Orbits::j2): node and perigee rates and
+    // the axis ratios that rotate the (aP, bQ) frame in its plane
+    kDOm = 40, kDw = 41,             // dOmega/dt, domega/dt [rad/s]
+    kBA = 42, kAB = 43,              // b/a, a/b
+    kNCol = 44
 };
+
+// J2 secular propagator constants (EGM-96 / WGS-84, reading R19)
+constexpr double kJ2 = 1.08262668e-3;
+constexpr double kRe = 6378.137;   // km
 
 // Contour point count (N_it) per eccentricity class (reading R15)
 __host__ __device__ constexpr int class_points(int cls)
@@ -45,6 +53,7 @@ struct Orbits {
     const uint8_t* cls;  // eccentricity class per object
     int64_t n;
     int64_t n0;          // objects [0, n0) are class 0 (records sorted by class)
+    int j2;              // 1: J2 secular propagator (plane and perigee rotate; columns kDOm..kAB)
     // records are streamed once per step: evict-first so they do not push the per-step grid
     // (slots, bitmap, entries) out of L2
     __device__ __forceinline__ double at(int c, int64_t r) const { return __ldcs(rec + c * n + r); }
@@ -280,8 +289,14 @@ __device__ __forceinline__ void kepler_solve(double M, double e, int cls, const 
 
 // Position (and velocity) of object r at time t.
 //   r = (cos E - e) aP + sin E bQ;     v = n/(1 - e cos E) (-sin E aP + cos E bQ)
+// J2 secular (O.j2): the epoch frame (P, Q) turns by domega t about the orbit normal h and the
+// plane by dOmega t about z.  With X = cos E - e, Y = sin E, the in-plane coordinates become
+//   r = [X cw - (b/a) Y sw] aP + [(a/b) X sw + Y cw] bQ,   (cw, sw) = cos, sin(domega t)
+// followed by the z-rotation; velocity = the rotated two-body velocity + domega h x r (in the
+// plane: (x, y) -> (-y, x)) + dOmega z x r.
 // kClass: 0 = object known to be class 0 (lean path), -1 = any class
-template <bool kVel, int kClass = -1>
+// kJ2: 0 = two-body only, 1 = J2 secular only, -1 = per O.j2 (runtime, warp-uniform)
+template <bool kVel, int kClass = -1, int kJ2 = -1>
 __device__ __forceinline__ void state(const Orbits& O, int64_t r, double t, double p[3], double v[3])
 {
     const double e = O.at(kE, r);
@@ -289,15 +304,53 @@ __device__ __forceinline__ void state(const Orbits& O, int64_t r, double t, doub
     double E, sE, cE;
     if (kClass == 0) contour_core<4>(M, e, O, r, E, sE, cE);
     else kepler_solve(M, e, O.cls[r], O, r, E, sE, cE);
-    const double x = cE - e;
+    double x = cE - e, y = sE;              // coefficients of aP and bQ
+    double vx = -sE, vy = cE;               // velocity coefficients (times n/(1 - e cos E))
+    const bool j2 = kJ2 == 1 || (kJ2 == -1 && O.j2);
+    double sO = 0.0, cO = 1.0, dOm = 0.0, dw = 0.0, ba = 1.0, ab = 1.0;
+    if (j2) {
+        dOm = O.at(kDOm, r);
+        dw = O.at(kDw, r);
+        ba = O.at(kBA, r);
+        ab = O.at(kAB, r);
+        double sw, cw;
+        sincos_fast(dw * t, sw, cw);
+        sincos_fast(dOm * t, sO, cO);
+        const double xr = fma(x, cw, -ba * y * sw), yr = fma(ab * x, sw, y * cw);
+        x = xr;
+        y = yr;
+        if (kVel) {
+            const double vxr = fma(vx, cw, -ba * vy * sw), vyr = fma(ab * vx, sw, vy * cw);
+            vx = vxr;
+            vy = vyr;
+        }
+    }
     const double ap[3] = {O.at(kAPx, r), O.at(kAPy, r), O.at(kAPz, r)};
     const double bq[3] = {O.at(kBQx, r), O.at(kBQy, r), O.at(kBQz, r)};
 #pragma unroll
-    for (int c = 0; c < 3; ++c) p[c] = fma(x, ap[c], sE * bq[c]);
+    for (int c = 0; c < 3; ++c) p[c] = fma(x, ap[c], y * bq[c]);
     if (kVel) {
         const double k = O.at(kNm, r) / fma(-e, cE, 1.0);
+        if (j2) {
+            // domega h x r: the in-plane vector (X, Y) in unit (P, Q) axes turns to (-Y, X);
+            // in (aP, bQ) coefficients: (-(b/a) y, (a/b) x)
+            const double wx = k * vx - dw * ba * y, wy = k * vy + dw * ab * x;
 #pragma unroll
-        for (int c = 0; c < 3; ++c) v[c] = k * fma(-sE, ap[c], cE * bq[c]);
+            for (int c = 0; c < 3; ++c) v[c] = fma(wx, ap[c], wy * bq[c]);
+        } else {
+#pragma unroll
+            for (int c = 0; c < 3; ++c) v[c] = k * fma(vx, ap[c], vy * bq[c]);
+        }
+    }
+    if (j2) {   // plane rotation about z by dOmega t (and dOmega z x r for the velocity)
+        const double px = fma(p[0], cO, -p[1] * sO), py = fma(p[0], sO, p[1] * cO);
+        p[0] = px;
+        p[1] = py;
+        if (kVel) {
+            const double qx = fma(v[0], cO, -v[1] * sO), qy = fma(v[0], sO, v[1] * cO);
+            v[0] = fma(-dOm, py, qx);
+            v[1] = fma(dOm, px, qy);
+        }
     }
 }
 

@@ -74,7 +74,7 @@ __global__ void k_classify(Elements el, int64_t n, uint32_t* key, uint32_t* idx,
 }
 
 __global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, int64_t n,
-                                double* __restrict__ rec, uint8_t* __restrict__ cls)
+                                double* __restrict__ rec, uint8_t* __restrict__ cls, int j2)
 {
     const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (r >= n) return;
@@ -96,7 +96,23 @@ __global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, 
     const double M0 = E0 - e * sin(E0);
     auto put = [&](int c, double v) { rec[c * n + r] = v; };
     put(kM0, M0);
-    put(kNm, sqrt(kMu / (a * a * a)));
+    const double n0 = sqrt(kMu / (a * a * a));
+    if (j2) {
+        // J2 secular rates (Vallado & McClain [41] Sec. 9.6):
+        //   k = J2 (R_E / p)^2, p = a (1 - e^2)
+        //   dM/dt = n0 [1 + 1.5 k sqrt(1 - e^2) (1 - 1.5 sin^2 i)], dOmega/dt = -1.5 n0 k cos i,
+        //   domega/dt = 0.75 n0 k (4 - 5 sin^2 i)
+        const double sq = sqrt((1.0 - e) * (1.0 + e));
+        const double rp = kRe / (a * (1.0 - e) * (1.0 + e));
+        const double k = kJ2 * rp * rp;
+        put(kNm, n0 * (1.0 + 1.5 * k * sq * (1.0 - 1.5 * si * si)));
+        put(kDOm, -1.5 * n0 * k * ci);
+        put(kDw, 0.75 * n0 * k * (4.0 - 5.0 * si * si));
+        put(kBA, sq);
+        put(kAB, 1.0 / sq);
+    } else {
+        put(kNm, n0);
+    }
     put(kE, e);
     put(kAPx, a * P[0]); put(kAPy, a * P[1]); put(kAPz, a * P[2]);
     put(kBQx, b * Q[0]); put(kBQy, b * Q[1]); put(kBQz, b * Q[2]);
@@ -142,9 +158,9 @@ cudaError_t launch_classify(const Elements& el, int64_t n, uint32_t* key, uint32
 }
 
 cudaError_t launch_build_records(const Elements& el, const uint32_t* perm, int64_t n, double* rec,
-                                 uint8_t* cls, cudaStream_t st, LaunchCount& lc)
+                                 uint8_t* cls, int j2, cudaStream_t st, LaunchCount& lc)
 {
-    k_build_records<<<blocks_for(n, 128), 128, 0, st>>>(el, perm, n, rec, cls);
+    k_build_records<<<blocks_for(n, 128), 128, 0, st>>>(el, perm, n, rec, cls, j2);
     lc.bump();
     return cudaGetLastError();
 }
@@ -190,7 +206,7 @@ cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long l
 // (Eq. 2) and its occupancy bitmap; the entry {x, y, z, next} (Fig. 6) is
 // written once, coalesced.  kClass0: objects [0, n0) (e <= 0.01: lean N = 4 Contour path).
 // ---------------------------------------------------------------------------------------
-template <bool kClass0, bool kChained>
+template <bool kClass0, bool kChained, int kJ2>
 __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, const GridTab& tab,
                                          Entry* __restrict__ ents, uint64_t mask, int64_t k0, int s,
                                          int64_t r, double t0, double dt, uint32_t tag, Ctrl* ctrl)
@@ -200,7 +216,7 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
 #ifdef CD_ABL_NO_PROP   // ablation (timing experiments only): position from one record column
     p[0] = O.at(kAPx, r) + t; p[1] = O.at(kAPy, r); p[2] = O.at(kAPz, r);
 #else
-    state<false, kClass0 ? 0 : -1>(O, r, t, p, v);
+    state<false, kClass0 ? 0 : -1, kJ2>(O, r, t, p, v);
 #endif
     int c[3];
     uint32_t next = kNil, ctag = 0;
@@ -516,7 +532,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
 #ifndef CD_STEP_MINB
 #define CD_STEP_MINB 6
 #endif
-template <bool kChained>
+template <bool kChained, int kJ2>
 __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
 {
     const uint32_t bx = blockIdx.x;
@@ -535,14 +551,14 @@ __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
         const int s = (int)(bx / nbA);
         const int64_t r = (int64_t)(bx % nbA) * 256 + threadIdx.x;
         if (r < a.O.n0)
-            do_build<true, kChained>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
+            do_build<true, kChained, kJ2>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
                                      a.dt, a.build_tag, a.ctrl);
     } else if (bx < nA + nB) {
         const uint32_t b2 = bx - nA;
         const int s = (int)(b2 / nbB);
         const int64_t r = a.O.n0 + (int64_t)(b2 % nbB) * 256 + threadIdx.x;
         if (r < a.O.n)
-            do_build<false, kChained>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
+            do_build<false, kChained, kJ2>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
                                       a.dt, a.build_tag, a.ctrl);
     } else {
         const uint32_t b3 = bx - nA - nB;
@@ -582,8 +598,13 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
     const int64_t blocks = a.build_B * (a.nbA + a.nbB) + a.nCblocks;
     if (blocks == 0) return cudaSuccess;
     lc.bump();
-    if (a.chained) return launch_ex(k_step<true>, dim3((unsigned)blocks), dim3(256), st, win, a.pdl != 0, a);
-    return launch_ex(k_step<false>, dim3((unsigned)blocks), dim3(256), st, win, false, a);
+    if (a.O.j2) {   // J2 secular propagator: the rotation is compiled into its own instances
+        if (a.chained)
+            return launch_ex(k_step<true, 1>, dim3((unsigned)blocks), dim3(256), st, win, a.pdl != 0, a);
+        return launch_ex(k_step<false, 1>, dim3((unsigned)blocks), dim3(256), st, win, false, a);
+    }
+    if (a.chained) return launch_ex(k_step<true, 0>, dim3((unsigned)blocks), dim3(256), st, win, a.pdl != 0, a);
+    return launch_ex(k_step<false, 0>, dim3((unsigned)blocks), dim3(256), st, win, false, a);
 }
 
 // ---------------------------------------------------------------------------------------

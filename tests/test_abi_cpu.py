@@ -43,7 +43,7 @@ def test_exports_every_declared_symbol(cds):
 
 
 def test_version_status_options(cds):
-    assert cds.cd_abi_version() == 1
+    assert cds.cd_abi_version() == 2
     assert cds.status_str(cds.CD_EINVAL) == "CD_EINVAL"
     assert cds.status_str(cds.CD_ENODEV) == "CD_ENODEV"
     o = cds.cd_options()
