@@ -103,6 +103,9 @@ def _bind_hybrid(L):
     L.orc_hybrid.argtypes = [P(_Elements), C.c_int64, C.c_double, C.c_double, C.c_double,
                              C.c_double, C.c_double, C.c_int64, C.c_int64, P(C.c_void_p),
                              P(C.c_int64)]
+    L.orc_legacy.restype = C.c_int64
+    L.orc_legacy.argtypes = [P(_Elements), C.c_int64, C.c_double, C.c_double, C.c_double,
+                             C.c_double, P(C.c_void_p), P(C.c_int64)]
     L.orc_pair_filter.restype = C.c_int
     L.orc_pair_filter.argtypes = [P(_Elements), C.c_int64, C.c_int64, C.c_double, C.c_double,
                                   C.c_double, P(C.c_double), C.c_int, P(C.c_int)]
@@ -251,6 +254,21 @@ def hybrid(pop, t0, t1, dt, d, v_margin=7.8, k_begin=0, k_end=-1):
     counts = (C.c_int64 * 6)()
     c = lib().orc_hybrid(P.ref, P.n, t0, t1, dt, d, gc, k_begin, k_end, C.byref(out), counts)
     keys = ("candidates", "ap_rejected", "coplanar", "path_rejected", "time_rejected", "window_work")
+    return _take(out, c, CONJ_DTYPE), dict(zip(keys, list(counts)))
+
+
+def legacy(pop, t0, t1, dt, d):
+    """Legacy full-window filter chain (O5): every pair through AP ->
+    coplanar -> orbit path -> time filter over [t0, t1], every local minimum of D below d in the
+    surviving intervals.  Returns (conjunctions, counts) with counts = pairs, ap_rejected,
+    coplanar, path_rejected, time_rejected, intervals."""
+    P = _Pop(pop)
+    if P.model:
+        raise ValueError("the orbital filters assume fixed orbit planes: Kepler propagator only")
+    out = C.c_void_p()
+    counts = (C.c_int64 * 6)()
+    c = lib().orc_legacy(P.ref, P.n, float(t0), float(t1), float(dt), float(d), C.byref(out), counts)
+    keys = ("pairs", "ap_rejected", "coplanar", "path_rejected", "time_rejected", "intervals")
     return _take(out, c, CONJ_DTYPE), dict(zip(keys, list(counts)))
 
 

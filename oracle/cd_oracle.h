@@ -50,6 +50,8 @@ int     orc_pair_filter(const orc_elements* el, int64_t i, int64_t j, double d, 
                         double thi, double* iv, int cap, int* niv);
 int64_t orc_hybrid(const orc_elements* el, int64_t n, double t0, double t1, double dt, double d,
                    double gc, int64_t k_begin, int64_t k_end, void** out, int64_t* counts);
+int64_t orc_legacy(const orc_elements* el, int64_t n, double t0, double t1, double dt, double d,
+                   void** out, int64_t* counts);
 void    orc_free(void* p);
 
 #ifdef __cplusplus

@@ -315,3 +315,204 @@ int64_t orc_hybrid(const orc_elements* el, int64_t n, double t0, double t1, doub
     *out = res;
     return total;
 }
+
+/* ------------------------------------------------------------------------------------------
+ * O5: legacy full-window filter chain.  The paper's comparison baseline
+ * screens every pair with the "classical orbital filters" alone, without a grid (P:43, P:189,
+ * P:315-318 accuracy comparison, "not possible with the legacy variant to calculate more
+ * than 64,000 satellites").  Per pair i < j, the O4 formulas over the whole window [t0, t1]:
+ *   AP -> coplanar (search all of [t0, t1]) -> orbit path -> time filter: every window of A at a
+ *   surviving node intersected with every window of B at the same node (both lists are sorted
+ *   in time and each object's windows are disjoint, so a merge visits each once)
+ * Conjunctions: every local minimum of D below d inside the intervals = every - -> + sign
+ * change of g = dr.dv sampled at spacing <= dt/8 (at least 8 samples per interval), bisected
+ * to 1e-10 s, with D < d and TCA in [t0, t1].  Each row is labelled with the nearest step
+ * k = floor((TCA - t0)/dt + 1/2) (reading R9); MULTI flags a second sign change within 2 dt
+ * (two minima the method's per-sample search may not separate); COPLANAR the coplanar path.
+ * Degenerate pairs (g identically 0) have no sign change and are not reported.
+ * counts: pairs, ap_rejected, coplanar, path_rejected, time_rejected, intervals.
+ * ------------------------------------------------------------------------------------------ */
+
+typedef struct {
+    double* v;
+    int64_t n, cap;
+} lg_buf;
+
+static void lg_push(lg_buf* b, double x, double y)
+{
+    if (b->n + 2 > b->cap) {
+        b->cap = b->cap ? 2 * b->cap : 64;
+        b->v = (double*)realloc(b->v, sizeof(double) * (size_t)b->cap);
+    }
+    b->v[b->n++] = x;
+    b->v[b->n++] = y;
+}
+
+/* every window of object o at node direction fc (half-angle al) within [t0, t1], in time order */
+static void lg_windows(const hy_orbit* o, double fc, double al, double t0, double t1, lg_buf* out)
+{
+    out->n = 0;
+    double Ml = hy_mean_of_true(fc - al, o->e);
+    double Mh = hy_mean_of_true(fc + al, o->e);
+    if (Mh < Ml) Mh += HY_TWO_PI;
+    double T = HY_TWO_PI / o->nmean;
+    double tl = (Ml - o->M0) / o->nmean, th = (Mh - o->M0) / o->nmean;
+    double kmin = floor((t0 - th) / T), kmax = ceil((t1 - tl) / T);
+    for (double k = kmin; k <= kmax; k += 1.0) {
+        double a = tl + k * T, b = th + k * T;
+        if (b < t0 || a > t1) continue;
+        lg_push(out, fmax(a, t0), fmin(b, t1));
+    }
+}
+
+/* filter chain of one pair over [t0, t1]; intervals appended to iv */
+static int lg_filter(const hy_orbit* A, const hy_orbit* B, double d, double t0, double t1,
+                     lg_buf* iv, lg_buf* wa, lg_buf* wb)
+{
+    iv->n = 0;
+    if (fmax(A->q, B->q) - fmin(A->Q, B->Q) > d) return ORC_H_AP;
+    double c[3] = {A->h[1] * B->h[2] - A->h[2] * B->h[1], A->h[2] * B->h[0] - A->h[0] * B->h[2],
+                   A->h[0] * B->h[1] - A->h[1] * B->h[0]};
+    double sD = sqrt(hy_dot(c, c));
+    double sA = sD > 0.0 ? d / (A->q * sD) : 2.0;
+    double sB = sD > 0.0 ? d / (B->q * sD) : 2.0;
+    int coplanar = sA >= 1.0 || sB >= 1.0;
+    double aA = 0.0, aB = 0.0;
+    if (!coplanar) {
+        aA = asin(sA);
+        aB = asin(sB);
+        coplanar = A->q * cos(aA) + B->q * cos(aB) <= d;
+    }
+    if (coplanar) {
+        lg_push(iv, t0, t1);
+        return ORC_H_COPLANAR;
+    }
+    double nn[3] = {c[0] / sD, c[1] / sD, c[2] / sD};
+    double fA = atan2(hy_dot(nn, A->Qv), hy_dot(nn, A->P));
+    double fB = atan2(hy_dot(nn, B->Qv), hy_dot(nn, B->P));
+    int any = 0;
+    for (int node = 0; node < 2; ++node) {
+        double off = node ? HY_PI : 0.0;
+        double rAl, rAh, rBl, rBh;
+        hy_radius_range(A, fA + off - aA, fA + off + aA, &rAl, &rAh);
+        hy_radius_range(B, fB + off - aB, fB + off + aB, &rBl, &rBh);
+        if (fmax(rAl, rBl) - fmin(rAh, rBh) > d) continue;   /* orbit path */
+        any = 1;
+        lg_windows(A, fA + off, aA, t0, t1, wa);
+        lg_windows(B, fB + off, aB, t0, t1, wb);
+        int64_t x = 0, y = 0;
+        while (x < wa->n && y < wb->n) {
+            double lo = fmax(wa->v[x], wb->v[y]), hi = fmin(wa->v[x + 1], wb->v[y + 1]);
+            if (hi > lo) lg_push(iv, lo, hi);
+            if (wa->v[x + 1] < wb->v[y + 1]) x += 2;
+            else y += 2;
+        }
+    }
+    if (!any) return ORC_H_PATH;
+    if (iv->n == 0) return ORC_H_TIME;
+    return 0;
+}
+
+int64_t orc_legacy(const orc_elements* el, int64_t n, double t0, double t1, double dt, double d,
+                   void** out, int64_t* counts)
+{
+    if (el->model != ORC_PROP_KEPLER) {   /* the filters assume fixed orbit planes (Kepler) */
+        *out = NULL;
+        return -1;
+    }
+    hy_orbit* o = (hy_orbit*)malloc(sizeof(hy_orbit) * (size_t)(n > 0 ? n : 1));
+    for (int64_t i = 0; i < n; ++i) hy_make(el, i, &o[i]);
+    int nt = orc_num_threads();
+    orc_conjunction** bufs = (orc_conjunction**)calloc((size_t)nt, sizeof(void*));
+    int64_t* bn = (int64_t*)calloc((size_t)nt, sizeof(int64_t));
+    int64_t* bc = (int64_t*)calloc((size_t)nt, sizeof(int64_t));
+    int64_t st[6] = {0, 0, 0, 0, 0, 0};
+#pragma omp parallel
+    {
+#ifdef _OPENMP
+        int tid = omp_get_thread_num();
+#else
+        int tid = 0;
+#endif
+        int64_t ls[6] = {0, 0, 0, 0, 0, 0};
+        lg_buf iv = {0}, wa = {0}, wb = {0}, mins = {0};
+#pragma omp for schedule(dynamic, 1)
+        for (int64_t i = 0; i < n; ++i) {
+            for (int64_t j = i + 1; j < n; ++j) {
+                ls[0]++;
+                int fl = lg_filter(&o[i], &o[j], d, t0, t1, &iv, &wa, &wb);
+                if (fl == ORC_H_AP) { ls[1]++; continue; }
+                if (fl == ORC_H_PATH) { ls[3]++; continue; }
+                if (fl == ORC_H_TIME) { ls[4]++; continue; }
+                if (fl == ORC_H_COPLANAR) ls[2]++;
+                ls[5] += iv.n / 2;
+                /* every - -> + sign change of g in the intervals: (tca, D) in mins */
+                mins.n = 0;
+                for (int64_t w = 0; w < iv.n; w += 2) {
+                    double lo = iv.v[w], hi = iv.v[w + 1];
+                    int64_t ns = (int64_t)ceil((hi - lo) / (dt / 8.0));
+                    if (ns < 8) ns = 8;
+                    double tprev = lo, gprev = hy_g(el, i, j, lo, NULL);
+                    for (int64_t s = 1; s <= ns; ++s) {
+                        double t = lo + (hi - lo) * (double)s / (double)ns;
+                        double g = hy_g(el, i, j, t, NULL);
+                        if (gprev < 0.0 && g >= 0.0) {
+                            double a = tprev, b = t;
+                            for (int it = 0; it < 200 && b - a > 1e-10; ++it) {
+                                double m = 0.5 * (a + b);
+                                if (hy_g(el, i, j, m, NULL) < 0.0) a = m;
+                                else b = m;
+                            }
+                            double tm = 0.5 * (a + b), D;
+                            hy_g(el, i, j, tm, &D);
+                            lg_push(&mins, tm, D);
+                        }
+                        tprev = t;
+                        gprev = g;
+                    }
+                }
+                for (int64_t x = 0; x < mins.n; x += 2) {
+                    double tm = mins.v[x], D = mins.v[x + 1];
+                    if (!(D < d) || tm < t0 || tm > t1) continue;
+                    uint32_t flags = fl == ORC_H_COPLANAR ? ORC_COPLANAR : 0u;
+                    for (int64_t y = 0; y < mins.n; y += 2)
+                        if (y != x && fabs(mins.v[y] - tm) < 2.0 * dt) flags |= ORC_MULTI;
+                    if (bn[tid] == bc[tid]) {
+                        bc[tid] = bc[tid] ? 2 * bc[tid] : 256;
+                        bufs[tid] = (orc_conjunction*)realloc(bufs[tid], sizeof(orc_conjunction) * (size_t)bc[tid]);
+                    }
+                    orc_conjunction* r = &bufs[tid][bn[tid]++];
+                    r->i = (uint32_t)i;
+                    r->j = (uint32_t)j;
+                    r->step = (uint32_t)floor((tm - t0) / dt + 0.5);
+                    r->flags = flags;
+                    r->tca = tm;
+                    r->pca = D;
+                }
+            }
+        }
+        free(iv.v);
+        free(wa.v);
+        free(wb.v);
+        free(mins.v);
+#pragma omp critical
+        for (int q = 0; q < 6; ++q) st[q] += ls[q];
+    }
+    int64_t total = 0;
+    for (int q = 0; q < nt; ++q) total += bn[q];
+    orc_conjunction* res = (orc_conjunction*)malloc(sizeof(orc_conjunction) * (size_t)(total > 0 ? total : 1));
+    int64_t off = 0;
+    for (int q = 0; q < nt; ++q) {
+        if (bn[q]) memcpy(res + off, bufs[q], sizeof(orc_conjunction) * (size_t)bn[q]);
+        off += bn[q];
+        free(bufs[q]);
+    }
+    free(bufs);
+    free(bn);
+    free(bc);
+    free(o);
+    qsort(res, (size_t)total, sizeof(orc_conjunction), hy_cmp);
+    for (int q = 0; q < 6; ++q) counts[q] = st[q];
+    *out = res;
+    return total;
+}
