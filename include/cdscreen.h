@@ -70,7 +70,15 @@ typedef enum {
 
 typedef enum {
     CD_GRID = 0,   /* grid-based variant                               */
-    CD_HYBRID = 1  /* hybrid: coarse grid + orbital filter chain             */
+    CD_HYBRID = 1, /* hybrid: coarse grid + orbital filter chain             */
+    CD_LEGACY = 2  /* legacy full-window filter chain, no grid (P:43 filters, P:189 legacy variant,
+                      P:315-318 accuracy comparison): every pair i < j passes apogee/perigee ->
+                      coplanarity -> orbit path -> time windows over all of [t0, t1] (coplanar
+                      pairs: all of [t0, t1]); the steps t_k inside the surviving intervals are
+                      sampled and every minimum below d reported by its owner step, with no Eq. 1
+                      speed assumption (gate d + (v_p,i + v_p,j) dt/2, perigee speeds): a superset
+                      of CD_GRID's result.  O(n^2) pairs; cd_screen/cd_screen_ex only, Kepler
+                      propagator only; pairs are split across ranks (n_ranks)                   */
 } cd_mode;
 
 /* Kepler elements, structure of arrays.  a > 0 [km], 0 <= e < 1, angles finite [rad]. */

@@ -327,7 +327,8 @@ int64_t orc_hybrid(const orc_elements* el, int64_t n, double t0, double t1, doub
  * Conjunctions: every local minimum of D below d inside the intervals = every - -> + sign
  * change of g = dr.dv sampled at spacing <= dt/8 (at least 8 samples per interval), bisected
  * to 1e-10 s, with D < d and TCA in [t0, t1].  Each row is labelled with the nearest step
- * k = floor((TCA - t0)/dt + 1/2) (reading R9); MULTI flags a second sign change within 2 dt
+ * k = floor((TCA - t0)/dt + 1/2) (reading R9) and, as in the grid variant, reported only if that
+ * step exists (k < K, reading R4); MULTI flags a second sign change within 2 dt
  * (two minima the method's per-sample search may not separate); COPLANAR the coplanar path.
  * Degenerate pairs (g identically 0) have no sign change and are not reported.
  * counts: pairs, ap_rejected, coplanar, path_rejected, time_rejected, intervals.
@@ -422,6 +423,7 @@ int64_t orc_legacy(const orc_elements* el, int64_t n, double t0, double t1, doub
     }
     hy_orbit* o = (hy_orbit*)malloc(sizeof(hy_orbit) * (size_t)(n > 0 ? n : 1));
     for (int64_t i = 0; i < n; ++i) hy_make(el, i, &o[i]);
+    const double K = (double)orc_num_steps(t0, t1, dt);
     int nt = orc_num_threads();
     orc_conjunction** bufs = (orc_conjunction**)calloc((size_t)nt, sizeof(void*));
     int64_t* bn = (int64_t*)calloc((size_t)nt, sizeof(int64_t));
@@ -474,6 +476,7 @@ int64_t orc_legacy(const orc_elements* el, int64_t n, double t0, double t1, doub
                 for (int64_t x = 0; x < mins.n; x += 2) {
                     double tm = mins.v[x], D = mins.v[x + 1];
                     if (!(D < d) || tm < t0 || tm > t1) continue;
+                    if (floor((tm - t0) / dt + 0.5) >= K) continue;   /* owner step beyond the last */
                     uint32_t flags = fl == ORC_H_COPLANAR ? ORC_COPLANAR : 0u;
                     for (int64_t y = 0; y < mins.n; y += 2)
                         if (y != x && fabs(mins.v[y] - tm) < 2.0 * dt) flags |= ORC_MULTI;

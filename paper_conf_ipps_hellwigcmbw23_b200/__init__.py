@@ -19,7 +19,7 @@ PKG = Path(__file__).resolve().parent
 LIB_PATH = PKG / "libcdscreen.so"
 
 CD_OK, CD_EINVAL, CD_ENOMEM, CD_ECUDA, CD_ENCCL, CD_ERANGE, CD_EINTERNAL, CD_ENODEV = range(8)
-CD_GRID, CD_HYBRID = 0, 1
+CD_GRID, CD_HYBRID, CD_LEGACY = 0, 1, 2
 CD_PROP_KEPLER, CD_PROP_J2 = 0, 1
 PROPAGATORS = {"kepler": CD_PROP_KEPLER, "j2": CD_PROP_J2}
 CD_FLAG_DEGENERATE = 2
@@ -260,7 +260,7 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
 
 def _mode(mode):
     if isinstance(mode, str):
-        return {"grid": CD_GRID, "hybrid": CD_HYBRID}[mode]
+        return {"grid": CD_GRID, "hybrid": CD_HYBRID, "legacy": CD_LEGACY}[mode]
     return int(mode)
 
 

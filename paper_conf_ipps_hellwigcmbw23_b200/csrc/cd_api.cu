@@ -26,6 +26,7 @@
 #include "../../include/cdscreen.h"
 #include "cd_internal.h"
 #include "cd_hybrid.h"
+#include "cd_legacy.h"
 
 using namespace cdk;
 using namespace cdh;
@@ -1064,6 +1065,81 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     return CD_OK;
 }
 
+// Legacy full-window filter chain (mode CD_LEGACY, cd_legacy.cu): the
+// n(n-1)/2 pairs are filtered in chunks; each chunk's intervals are searched before the next
+// chunk is filtered.  A chunk whose work items or records overflow is redone with larger
+// buffers (device counters restored first).  Ranks share the pairs by contiguous ranges.
+cd_status run_legacy(Call& C, const OrbitSet& S, double t0, double t1, double dt, double d,
+                     const cd_options& o, int64_t K, Result& R, cd_stats& stats)
+{
+    cudaStream_t st = C.st;
+    const Orbits O = S.view();
+    const int64_t n = O.n;
+    const unsigned __int128 total = n >= 2 ? (unsigned __int128)n * (unsigned __int128)(n - 1) / 2 : 0;
+    const uint64_t pb = (uint64_t)(total * (unsigned)o.rank / (unsigned)o.n_ranks);
+    const uint64_t pe = (uint64_t)(total * (unsigned)(o.rank + 1) / (unsigned)o.n_ranks);
+    stats.steps = (uint64_t)K;
+    stats.object_steps = (uint64_t)K * (uint64_t)n;
+    stats.candidates = pe - pb;   // pairs screened by this rank
+    if (pe <= pb) return CD_OK;
+    LegacyParams P{t0, t1, dt, d, K};
+    DBuf<unsigned char> hrec(st);
+    CU(hrec.alloc(hybrid_record_bytes() * (size_t)n));
+    CU(launch_build_hybrid_records(O, hrec.p, st, C.lc));
+    DBuf<Ctrl> ctrl(st);
+    CU(ctrl.alloc(1));
+    CU(cudaMemsetAsync(ctrl.p, 0, sizeof(Ctrl), st));
+    DBuf<unsigned long long> cnt(st);   // [0] work items, [1] next item of the search
+    CU(cnt.alloc(2));
+    size_t wcap = size_t(1) << 22;
+    DBuf<Work> w(st);
+    CU(w.alloc(wcap));
+    size_t ocap = size_t(1) << 20;
+    CU(R.conj.grow(ocap, 0, st));
+    Ctrl before{}, after{};
+    unsigned long long hw[2];
+    uint64_t chunk = uint64_t(1) << 26;
+    C.pt.start(kPhRefine);
+    for (uint64_t p0 = pb; p0 < pe;) {
+        const uint64_t p1 = std::min<uint64_t>(pe, p0 + chunk);
+        CU(cudaMemcpyAsync(&before, ctrl.p, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
+        CU(cudaMemsetAsync(cnt.p, 0, 2 * sizeof(unsigned long long), st));
+        CU(launch_legacy_filter(P, hrec.p, n, p0, p1, w.p, wcap, cnt.p, ctrl.p, st, C.lc));
+        CU(launch_legacy_search(O, P, hrec.p, w.p, cnt.p, wcap, cnt.p + 1, R.conj.p, ocap, ctrl.p, st,
+                                C.lc));
+        CU(cudaMemcpyAsync(hw, cnt.p, sizeof hw, cudaMemcpyDeviceToHost, st));
+        CU(cudaMemcpyAsync(&after, ctrl.p, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
+        CU(cudaStreamSynchronize(st));
+        const bool wover = hw[0] > wcap, oover = after.n_conj > ocap;
+        if (wover || oover) {   // redo the chunk with room for it
+            ++stats.retries;
+            if (wover) {
+                wcap = (size_t)(hw[0] * 1.25) + 1024;
+                CU(w.alloc(wcap));
+            }
+            if (oover) {
+                const size_t ncap = std::max<size_t>(2 * ocap, (size_t)(after.n_conj * 1.25) + 1024);
+                CU(R.conj.grow(ncap, before.n_conj, st));
+                ocap = ncap;
+            }
+            CU(cudaMemcpyAsync(ctrl.p, &before, sizeof(Ctrl), cudaMemcpyHostToDevice, st));
+            continue;
+        }
+        p0 = p1;
+        // keep a chunk's work items within the buffer: grow the chunk while they fill < 1/4
+        if (hw[0] < wcap / 4 && chunk < (uint64_t(1) << 34)) chunk *= 2;
+        else if (hw[0] > wcap / 2 && chunk > (uint64_t(1) << 16)) chunk /= 2;
+    }
+    C.pt.stop();
+    R.n_conj = (size_t)after.n_conj;
+    stats.refined = after.n_refined;
+    stats.hybrid_ap_rejected = after.n_ap;
+    stats.hybrid_coplanar = after.n_coplanar;
+    stats.hybrid_path_rejected = after.n_path;
+    stats.hybrid_time_rejected = after.n_time;
+    return CD_OK;
+}
+
 cd_options defaults()
 {
     cd_options o;
@@ -1079,9 +1155,10 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
     out->count = 0;
     out->_owner = nullptr;
     const cd_options o = opt ? *opt : defaults();
-    if (mode != CD_GRID && mode != CD_HYBRID) return fail(CD_EINVAL, "unknown mode %d", (int)mode);
-    if (mode == CD_HYBRID && o.propagator != CD_PROP_KEPLER)
-        return fail(CD_EINVAL, "CD_HYBRID needs CD_PROP_KEPLER (the filters assume fixed orbit planes)");
+    if (mode != CD_GRID && mode != CD_HYBRID && mode != CD_LEGACY)
+        return fail(CD_EINVAL, "unknown mode %d", (int)mode);
+    if (mode != CD_GRID && o.propagator != CD_PROP_KEPLER)
+        return fail(CD_EINVAL, "CD_HYBRID and CD_LEGACY need CD_PROP_KEPLER (the filters assume fixed orbit planes)");
     int64_t K = 0;
     TRY(validate_scalars(n, t0, t1, dt, d, o, &K));
     cd_stats stats;
@@ -1099,7 +1176,8 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
         if (n > 0) TRY(prepare_orbits(C, el, n, o, S));
         else if (!el) return fail(CD_EINVAL, "elements must be non-NULL");
         DBG("screen: orbits ready");
-        TRY(run(C, S, t0, t1, dt, d, mode, o, K, Want::Conj, R, stats));
+        if (mode == CD_LEGACY) TRY(run_legacy(C, S, t0, t1, dt, d, o, K, R, stats));
+        else TRY(run(C, S, t0, t1, dt, d, mode, o, K, Want::Conj, R, stats));
         DBG("screen: run done");
         if (R.n_conj) {
             C.pt.start(kPhFinalize);

@@ -1,0 +1,130 @@
+// cd_filters.cuh -- classical orbital filter geometry shared by the hybrid variant (cd_hybrid.cu,
+// coarse-step candidates) and the legacy full-window chain (cd_legacy.cu, all pairs): compact
+// per-object records and the apogee/perigee, orbit-path and time-filter formulas of reading R17
+// (PAPER.md:43 names the filters [13], [15]).
+#pragma once
+#include "cd_refine.cuh"
+
+namespace cdh {
+namespace filt {
+
+using namespace cdk;
+
+
+constexpr double kPiH = 3.14159265358979323846;
+constexpr double kTwoPiH = 6.28318530717958647692;
+
+struct __align__(128) HOrbit {   // one 128-byte line per object (compact gather in the filter)
+    double e, q, Q, p, nm, M0;
+    double P[3], Qv[3], h[3];
+    double pad;
+};
+static_assert(sizeof(HOrbit) == 128, "HOrbit must be one 128-byte line");
+
+__device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o)
+{
+    const double ap[3] = {O.at(kAPx, r), O.at(kAPy, r), O.at(kAPz, r)};
+    const double bq[3] = {O.at(kBQx, r), O.at(kBQy, r), O.at(kBQz, r)};
+    const double a = sqrt(ap[0] * ap[0] + ap[1] * ap[1] + ap[2] * ap[2]);
+    const double b = sqrt(bq[0] * bq[0] + bq[1] * bq[1] + bq[2] * bq[2]);
+    for (int c = 0; c < 3; ++c) {
+        o.P[c] = ap[c] / a;
+        o.Qv[c] = bq[c] / b;
+    }
+    o.h[0] = o.P[1] * o.Qv[2] - o.P[2] * o.Qv[1];
+    o.h[1] = o.P[2] * o.Qv[0] - o.P[0] * o.Qv[2];
+    o.h[2] = o.P[0] * o.Qv[1] - o.P[1] * o.Qv[0];
+    o.e = O.at(kE, r);
+    o.q = a * (1.0 - o.e);
+    o.Q = a * (1.0 + o.e);
+    o.p = a * (1.0 - o.e) * (1.0 + o.e);
+    o.nm = O.at(kNm, r);
+    o.M0 = O.at(kM0, r);
+    o.pad = 0.0;
+}
+
+// mean anomaly of true anomaly f, in [-pi, pi]: f is reduced to [-pi, pi] first so the half-angle
+// formula stays on its principal branch (window ends on different branches would cancel a window)
+__device__ __forceinline__ double mean_of_true(double f, double e)
+{
+    f = remainder(f, kTwoPiH);
+    double sf, cf;
+    sincos(0.5 * f, &sf, &cf);
+    const double E = 2.0 * atan2(sqrt(1.0 - e) * sf, sqrt(1.0 + e) * cf);
+    return E - e * sin(E);
+}
+
+// radius range over true anomalies [f1, f2], f2 - f1 < pi
+__device__ __forceinline__ void radius_range(const HOrbit& o, double f1, double f2, double& rmin,
+                                             double& rmax)
+{
+    const double r1 = o.p / (1.0 + o.e * cos(f1)), r2 = o.p / (1.0 + o.e * cos(f2));
+    rmin = fmin(r1, r2);
+    rmax = fmax(r1, r2);
+    if (ceil(f1 / kTwoPiH) * kTwoPiH <= f2) rmin = o.q;                  // perigee inside
+    if (kPiH + ceil((f1 - kPiH) / kTwoPiH) * kTwoPiH <= f2) rmax = o.Q;  // apogee inside
+}
+
+// first-occurrence time window [tl, th] (mod T) of true anomaly in (fc - al, fc + al)
+__device__ __forceinline__ void node_window(const HOrbit& o, double fc, double al, double& tl,
+                                            double& th)
+{
+    const double Ml = mean_of_true(fc - al, o.e);
+    double Mh = mean_of_true(fc + al, o.e);
+    if (Mh < Ml) Mh += kTwoPiH;
+    tl = (Ml - o.M0) / o.nm;
+    th = (Mh - o.M0) / o.nm;
+}
+
+// Pair geometry of the filter chain (reading R17).  Returns 1 if the apogee/perigee filter
+// rejects the pair; otherwise 0 with coplanar set, and for non-coplanar pairs the node-window
+// half-angles aA, aB and the true anomalies fA, fB of the mutual node line in each orbit.
+//   AP:        exclude iff max(q_A, q_B) - min(Q_A, Q_B) > d
+//   coplanar:  s_X = d / (q_X sin D) >= 1 for A or B, or q_A cos(asin s_A) + q_B cos(asin s_B) <= d
+__device__ __forceinline__ int pair_geometry(const HOrbit& A, const HOrbit& B, double d,
+                                             bool& coplanar, double& aA, double& aB, double& fA,
+                                             double& fB)
+{
+    if (fmax(A.q, B.q) - fmin(A.Q, B.Q) > d) return 1;
+    const double c[3] = {A.h[1] * B.h[2] - A.h[2] * B.h[1], A.h[2] * B.h[0] - A.h[0] * B.h[2],
+                         A.h[0] * B.h[1] - A.h[1] * B.h[0]};
+    const double sD = sqrt(c[0] * c[0] + c[1] * c[1] + c[2] * c[2]);
+    const double sA = sD > 0.0 ? d / (A.q * sD) : 2.0;
+    const double sB = sD > 0.0 ? d / (B.q * sD) : 2.0;
+    coplanar = sA >= 1.0 || sB >= 1.0;
+    aA = aB = fA = fB = 0.0;
+    if (!coplanar) {
+        aA = asin(sA);
+        aB = asin(sB);
+        coplanar = A.q * cos(aA) + B.q * cos(aB) <= d;
+    }
+    if (coplanar) return 0;
+    const double nn[3] = {c[0] / sD, c[1] / sD, c[2] / sD};
+    fA = atan2(nn[0] * A.Qv[0] + nn[1] * A.Qv[1] + nn[2] * A.Qv[2],
+               nn[0] * A.P[0] + nn[1] * A.P[1] + nn[2] * A.P[2]);
+    fB = atan2(nn[0] * B.Qv[0] + nn[1] * B.Qv[1] + nn[2] * B.Qv[2],
+               nn[0] * B.P[0] + nn[1] * B.P[1] + nn[2] * B.P[2]);
+    return 0;
+}
+
+// orbit-path filter at one mutual node (off = 0 or pi): true iff the radial ranges of A and B
+// over their node windows are more than d apart (|r_A - r_B| >= ||r_A| - |r_B||)
+__device__ __forceinline__ bool node_closed(const HOrbit& A, const HOrbit& B, double d, double fA,
+                                            double fB, double aA, double aB, double off)
+{
+    double rAl, rAh, rBl, rBh;
+    radius_range(A, fA + off - aA, fA + off + aA, rAl, rAh);
+    radius_range(B, fB + off - aB, fB + off + aB, rBl, rBh);
+    return fmax(rAl, rBl) - fmin(rAh, rBh) > d;
+}
+
+// warp-aggregated counter increment (one atomic per group of converged lanes)
+__device__ __forceinline__ void count1(unsigned long long* cnt)
+{
+    cg::coalesced_group g = cg::coalesced_threads();
+    if (g.thread_rank() == 0) atomicAdd(cnt, (unsigned long long)g.size());
+}
+
+
+}  // namespace filt
+}  // namespace cdh

@@ -19,78 +19,15 @@
 #ifdef CD_DEBUG_FILTER
 #include <cstdio>
 #endif
-#include "cd_refine.cuh"
+#include "cd_filters.cuh"
 
 using namespace cdk;
 
 namespace cdh {
 
+using namespace filt;
+
 namespace {
-
-constexpr double kPiH = 3.14159265358979323846;
-constexpr double kTwoPiH = 6.28318530717958647692;
-
-struct __align__(128) HOrbit {   // one 128-byte line per object (compact gather in the filter)
-    double e, q, Q, p, nm, M0;
-    double P[3], Qv[3], h[3];
-    double pad;
-};
-static_assert(sizeof(HOrbit) == 128, "HOrbit must be one 128-byte line");
-
-__device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o)
-{
-    const double ap[3] = {O.at(kAPx, r), O.at(kAPy, r), O.at(kAPz, r)};
-    const double bq[3] = {O.at(kBQx, r), O.at(kBQy, r), O.at(kBQz, r)};
-    const double a = sqrt(ap[0] * ap[0] + ap[1] * ap[1] + ap[2] * ap[2]);
-    const double b = sqrt(bq[0] * bq[0] + bq[1] * bq[1] + bq[2] * bq[2]);
-    for (int c = 0; c < 3; ++c) {
-        o.P[c] = ap[c] / a;
-        o.Qv[c] = bq[c] / b;
-    }
-    o.h[0] = o.P[1] * o.Qv[2] - o.P[2] * o.Qv[1];
-    o.h[1] = o.P[2] * o.Qv[0] - o.P[0] * o.Qv[2];
-    o.h[2] = o.P[0] * o.Qv[1] - o.P[1] * o.Qv[0];
-    o.e = O.at(kE, r);
-    o.q = a * (1.0 - o.e);
-    o.Q = a * (1.0 + o.e);
-    o.p = a * (1.0 - o.e) * (1.0 + o.e);
-    o.nm = O.at(kNm, r);
-    o.M0 = O.at(kM0, r);
-    o.pad = 0.0;
-}
-
-// mean anomaly of true anomaly f, in [-pi, pi]: f is reduced to [-pi, pi] first so the half-angle
-// formula stays on its principal branch (window ends on different branches would cancel a window)
-__device__ __forceinline__ double mean_of_true(double f, double e)
-{
-    f = remainder(f, kTwoPiH);
-    double sf, cf;
-    sincos(0.5 * f, &sf, &cf);
-    const double E = 2.0 * atan2(sqrt(1.0 - e) * sf, sqrt(1.0 + e) * cf);
-    return E - e * sin(E);
-}
-
-// radius range over true anomalies [f1, f2], f2 - f1 < pi
-__device__ __forceinline__ void radius_range(const HOrbit& o, double f1, double f2, double& rmin,
-                                             double& rmax)
-{
-    const double r1 = o.p / (1.0 + o.e * cos(f1)), r2 = o.p / (1.0 + o.e * cos(f2));
-    rmin = fmin(r1, r2);
-    rmax = fmax(r1, r2);
-    if (ceil(f1 / kTwoPiH) * kTwoPiH <= f2) rmin = o.q;                  // perigee inside
-    if (kPiH + ceil((f1 - kPiH) / kTwoPiH) * kTwoPiH <= f2) rmax = o.Q;  // apogee inside
-}
-
-// first-occurrence time window [tl, th] (mod T) of true anomaly in (fc - al, fc + al)
-__device__ __forceinline__ void node_window(const HOrbit& o, double fc, double al, double& tl,
-                                            double& th)
-{
-    const double Ml = mean_of_true(fc - al, o.e);
-    double Mh = mean_of_true(fc + al, o.e);
-    if (Mh < Ml) Mh += kTwoPiH;
-    tl = (Ml - o.M0) / o.nm;
-    th = (Mh - o.M0) / o.nm;
-}
 
 // the (at most one per period) copy of the periodic window [tl, th] + k T overlapping [lo, hi];
 // windows are shorter than half a period and [lo, hi] (one coarse cell) is far shorter than a
@@ -110,13 +47,6 @@ __device__ __forceinline__ int window_copies(double tl, double th, double T, dou
         }
     }
     return c;
-}
-
-// warp-aggregated counter increment (one atomic per group of converged lanes)
-__device__ __forceinline__ void count1(unsigned long long* cnt)
-{
-    cg::coalesced_group g = cg::coalesced_threads();
-    if (g.thread_rank() == 0) atomicAdd(cnt, (unsigned long long)g.size());
 }
 
 }  // namespace
@@ -143,34 +73,17 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
         const Cand cd = q[idx];
         const HOrbit A = hr[cd.i], B = hr[cd.j];
         const double d = P.d;
-        // apogee / perigee
-        if (fmax(A.q, B.q) - fmin(A.Q, B.Q) > d) {
+        bool coplanar;
+        double aA, aB, fA, fB;
+        if (pair_geometry(A, B, d, coplanar, aA, aB, fA, fB)) {   // apogee / perigee
             count1(&ctrl->n_ap);
             continue;
-        }
-        // mutual inclination and node line
-        const double c[3] = {A.h[1] * B.h[2] - A.h[2] * B.h[1], A.h[2] * B.h[0] - A.h[0] * B.h[2],
-                             A.h[0] * B.h[1] - A.h[1] * B.h[0]};
-        const double sD = sqrt(c[0] * c[0] + c[1] * c[1] + c[2] * c[2]);
-        const double sA = sD > 0.0 ? d / (A.q * sD) : 2.0;
-        const double sB = sD > 0.0 ? d / (B.q * sD) : 2.0;
-        bool coplanar = sA >= 1.0 || sB >= 1.0;
-        double aA = 0.0, aB = 0.0;
-        if (!coplanar) {
-            aA = asin(sA);
-            aB = asin(sB);
-            coplanar = A.q * cos(aA) + B.q * cos(aB) <= d;
         }
         if (coplanar) {   // same procedure as the grid-based variant
             count1(&ctrl->n_coplanar);
             grid_refine_item(O, P, cd, 4u /* CD_FLAG_COPLANAR */, w, wcap, n_work, out, ocap, ctrl);
             continue;
         }
-        const double nn[3] = {c[0] / sD, c[1] / sD, c[2] / sD};
-        const double fA = atan2(nn[0] * A.Qv[0] + nn[1] * A.Qv[1] + nn[2] * A.Qv[2],
-                                nn[0] * A.P[0] + nn[1] * A.P[1] + nn[2] * A.P[2]);
-        const double fB = atan2(nn[0] * B.Qv[0] + nn[1] * B.Qv[1] + nn[2] * B.Qv[2],
-                                nn[0] * B.P[0] + nn[1] * B.P[1] + nn[2] * B.P[2]);
         // owner cell of the coarse step, relative to t_k
         const double tk = fma((double)cd.step, P.dt, P.t0);
         const double lo = fmax(tk - 0.5 * P.dt, P.t0) - tk, hi = fmin(tk + 0.5 * P.dt, P.t1) - tk;
@@ -178,10 +91,7 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
         int nwin = 0;
         for (int node = 0; node < 2; ++node) {
             const double off = node ? kPiH : 0.0;
-            double rAl, rAh, rBl, rBh;
-            radius_range(A, fA + off - aA, fA + off + aA, rAl, rAh);
-            radius_range(B, fB + off - aB, fB + off + aB, rBl, rBh);
-            if (fmax(rAl, rBl) - fmin(rAh, rBh) > d) continue;   // orbit path: node closed
+            if (node_closed(A, B, d, fA, fB, aA, aB, off)) continue;   // orbit path: node closed
             any_node = true;
             double atl, ath, btl, bth;
             node_window(A, fA + off, aA, atl, ath);
@@ -203,8 +113,8 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
                 }
         }
 #ifdef CD_DEBUG_FILTER
-        printf("filter i=%u j=%u k=%u sD=%.17g sA=%.17g sB=%.17g fA=%.17g fB=%.17g lo=%g hi=%g any=%d nwin=%d A.M0=%.17g A.nm=%.17g B.M0=%.17g B.nm=%.17g\n",
-               cd.i, cd.j, cd.step, sD, sA, sB, fA, fB, lo, hi, (int)any_node, nwin, A.M0, A.nm, B.M0, B.nm);
+        printf("filter i=%u j=%u k=%u aA=%.17g aB=%.17g fA=%.17g fB=%.17g lo=%g hi=%g any=%d nwin=%d A.M0=%.17g A.nm=%.17g B.M0=%.17g B.nm=%.17g\n",
+               cd.i, cd.j, cd.step, aA, aB, fA, fB, lo, hi, (int)any_node, nwin, A.M0, A.nm, B.M0, B.nm);
 #endif
         if (!any_node) count1(&ctrl->n_path);
         else if (nwin == 0) count1(&ctrl->n_time);

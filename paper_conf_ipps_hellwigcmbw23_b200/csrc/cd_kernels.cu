@@ -643,92 +643,8 @@ __global__ void __launch_bounds__(128) k_brent(Orbits O, RefineParams P, const W
     for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < nw; idx += stride) {
         const Work it = w[idx];
         const double tk = fma((double)it.step, P.dt, P.t0);
-        double a = it.lo, b = it.hi;   // relative to t_k, already inside [t0, t1]
-        if (!(b > a)) continue;
-        const double lo = a, hi = b;
-        // Brent's localmin (golden section + successive parabolic interpolation)
-        const double cgold = 0.3819660112501051;   // (3 - sqrt 5)/2
-        const double eps = 1.4901161193847656e-08; // sqrt(2^-52)
-        const double tabs = 1e-9;                  // absolute tolerance in tau [s]
-        double x = a + cgold * (b - a), wv = x, vv = x;
-        double fx = dist2_at(O, it.i, it.j, tk + x), fw = fx, fv = fx;
-        double d = 0.0, e = 0.0;
-        for (int iter = 0; iter < 100; ++iter) {
-            const double m = 0.5 * (a + b);
-            const double tol = eps * fabs(x) + tabs;
-            const double t2 = 2.0 * tol;
-            if (fabs(x - m) <= t2 - 0.5 * (b - a)) break;
-            double pp = 0.0, qq = 0.0, rr = 0.0;
-            if (fabs(e) > tol) {
-                rr = (x - wv) * (fx - fv);
-                qq = (x - vv) * (fx - fw);
-                pp = (x - vv) * qq - (x - wv) * rr;
-                qq = 2.0 * (qq - rr);
-                if (qq > 0.0) pp = -pp;
-                else qq = -qq;
-                rr = e;
-                e = d;
-            }
-            if (fabs(pp) < fabs(0.5 * qq * rr) && pp > qq * (a - x) && pp < qq * (b - x)) {
-                d = pp / qq;
-                const double u = x + d;
-                if ((u - a) < t2 || (b - u) < t2) d = (x < m) ? tol : -tol;
-            } else {
-                e = (x < m) ? b - x : a - x;
-                d = cgold * e;
-            }
-            const double u = x + (fabs(d) >= tol ? d : (d > 0.0 ? tol : -tol));
-            const double fu = dist2_at(O, it.i, it.j, tk + u);
-            if (fu <= fx) {
-                if (u < x) b = x;
-                else a = x;
-                vv = wv; fv = fw; wv = x; fw = fx; x = u; fx = fu;
-            } else {
-                if (u < x) a = u;
-                else b = u;
-                if (fu <= fw || wv == x) {
-                    vv = wv; fv = fw; wv = u; fw = fu;
-                } else if (fu <= fv || vv == x || vv == wv) {
-                    vv = u; fv = fu;
-                }
-            }
-        }
-        // interval-edge rule
-        const double tol = eps * fabs(x) + tabs;
-        if (x - lo <= 3.0 * tol || hi - x <= 3.0 * tol) continue;
-        // polish: the minimum is the - -> + sign change of g = dr.dv = (1/2) dD^2/dtau.  Brent
-        // locates a flat minimum (slow relative motion) only to ~sqrt(eps) of D^2; bracket the
-        // root of g around x (expanding) and solve it by Illinois regula falsi to 1e-10 s
-        {
-            double hstep = fmax(4.0 * tol, 1e-6), d2a, d2b;
-            double ta = fmax(x - hstep, lo), tb = fmin(x + hstep, hi);
-            double ga = g_at(O, it.i, it.j, tk + ta, d2a), gb = g_at(O, it.i, it.j, tk + tb, d2b);
-            for (int ex = 0; ex < 12 && !(ga < 0.0 && gb >= 0.0); ++ex) {
-                hstep *= 4.0;
-                if (!(ga < 0.0)) { ta = fmax(x - hstep, lo); ga = g_at(O, it.i, it.j, tk + ta, d2a); }
-                if (!(gb >= 0.0)) { tb = fmin(x + hstep, hi); gb = g_at(O, it.i, it.j, tk + tb, d2b); }
-            }
-            if (ga < 0.0 && gb >= 0.0) {
-                int side = 0;
-                for (int k2 = 0; k2 < 80 && tb - ta > 1e-10; ++k2) {
-                    double tc = tb - gb * (tb - ta) / (gb - ga);
-                    if (!(tc > ta && tc < tb)) tc = 0.5 * (ta + tb);
-                    double d2c;
-                    const double gc = g_at(O, it.i, it.j, tk + tc, d2c);
-                    if (gc < 0.0) {
-                        ta = tc; ga = gc;
-                        if (side == -1) gb *= 0.5;
-                        side = -1;
-                    } else {
-                        tb = tc; gb = gc;
-                        if (side == 1) ga *= 0.5;
-                        side = 1;
-                    }
-                }
-                x = 0.5 * (ta + tb);
-                fx = dist2_at(O, it.i, it.j, tk + x);
-            }
-        }
+        double x, fx;
+        if (!brent_min(O, it.i, it.j, tk, it.lo, it.hi, x, fx)) continue;
         const double tca = tk + x;
         if (tca < P.t0 || tca > P.t1) continue;
         const double kstar = floor((tca - P.t0) / P.dt + 0.5);

@@ -86,3 +86,41 @@ def is_sorted(a):
     d = np.diff(k, axis=0)
     first = np.where(d[:, 0] != 0, d[:, 0], np.where(d[:, 1] != 0, d[:, 1], d[:, 2]))
     return bool(np.all(first >= 0))
+
+
+def _minima_near(pop, i, j, t_lo, t_hi, d):
+    """Local minima of D below d + 1 mm in [t_lo, t_hi] by 1 ms sampling (tie-break helper)."""
+    t = np.arange(t_lo, t_hi, 1e-3)
+    D, _ = oracle.pair_distance(pop, i, j, t)
+    return int(np.sum((D[1:-1] < D[:-2]) & (D[1:-1] <= D[2:]) & (D[1:-1] < d + MM)))
+
+
+def compare_legacy(pop, gpu, orc, t0, t1, dt, d):
+    """Legacy chain parity (oracle O5 vs CUDA): identical (i, j, step) sets and TCA/PCA, except
+    rows the oracle flags MULTI (a second minimum within 2 dt), |PCA - d| < 1 mm, TCA within
+    1e-3 s of an owner-cell boundary or of t0 / t1; a row on one side only must be explained by a
+    second minimum within 2 dt (1 ms sampling).  Returns dict(matched, excluded)."""
+    G = {(int(r["i"]), int(r["j"]), int(r["step"])): r for r in gpu}
+    O = {(int(r["i"]), int(r["j"]), int(r["step"])): r for r in orc}
+    assert len(G) == len(gpu), "duplicate rows in the GPU output"
+    matched = excluded = 0
+    for k in sorted(set(G) | set(O)):
+        g, o = G.get(k), O.get(k)
+        rows = [r for r in (g, o) if r is not None]
+        if (o is not None and o["flags"] & MULTI_FLAG) or any(_excluded_row(r, t0, t1, dt, d) for r in rows):
+            excluded += 1
+            continue
+        if g is None or o is None:
+            tk = t0 + k[2] * dt
+            n_min = _minima_near(pop, k[0], k[1], tk - 2 * dt, tk + 2 * dt, d)
+            assert n_min >= 2, (k, g, o, n_min)
+            excluded += 1
+            continue
+        assert abs(g["tca"] - o["tca"]) <= TCA_TOL, (k, g, o)
+        assert abs(g["pca"] - o["pca"]) <= PCA_TOL, (k, g, o)
+        assert (g["flags"] & 4) == (o["flags"] & 4), (k, g, o)
+        matched += 1
+    return {"matched": matched, "excluded": excluded}
+
+
+MULTI_FLAG = 1
