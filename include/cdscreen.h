@@ -160,6 +160,15 @@ typedef struct {
                                  exchange per object); 0 = default (2).  Results are identical. */
     cd_stats* stats;          /* optional output                                              */
     int propagator;           /* cd_propagator; default CD_PROP_KEPLER                        */
+    double shell_lo, shell_hi;/* radial shard [km] (object-space sharding for
+                                 populations whose per-step grid exceeds one GPU).  shell_hi = 0:
+                                 no shard (default).  Otherwise the call keeps exactly the
+                                 candidates whose smaller radius |r| at t_k lies in
+                                 [shell_lo, shell_hi) -- positions are bit-identical on every
+                                 shard, so the shards of a partition of [0, inf) report disjoint
+                                 sets whose union is the unsharded result -- provided the
+                                 elements passed are the shard's members (cd_shell_members: own
+                                 objects plus the g_c halo above the band).  CD_GRID/CD_HYBRID. */
 } cd_options;
 
 /* Fill *opt with the defaults above. */
@@ -227,6 +236,13 @@ typedef struct {
  * Validation as cd_screen (CD_EINVAL); out must be non-NULL. */
 cd_status cd_plan(size_t n, double t0, double t1, double dt, double d, cd_mode mode,
                   size_t mem_bytes, cd_plan_info* out);
+/* Members of the radial shard [shell_lo, shell_hi) (cd_options.shell_lo/hi): the indices i, in
+ * increasing order, whose radius range [a(1-e), a(1+e)] meets [shell_lo, shell_hi + gc) --
+ * every object that can be the nearer-to-Earth partner of a pair kept by the shard, or within
+ * g_c of one.  Host element pointers; idx is a caller-owned array of n entries; *count is set.
+ * Pure host arithmetic.  CD_EINVAL on NULL arguments, shell_hi <= shell_lo, invalid elements. */
+cd_status cd_shell_members(const cd_elements* el, size_t n, double shell_lo, double shell_hi,
+                           double gc, uint32_t* idx, size_t* count);
 void cd_candidates_free(cd_candidate* c);
 const char* cd_status_str(cd_status s);
 const char* cd_last_error(void);

@@ -33,7 +33,7 @@ CAND_DTYPE = np.dtype([("i", "<u4"), ("j", "<u4"), ("step", "<u4")])
 # C ABI symbols declared in include/cdscreen.h
 ABI_SYMBOLS = ("cd_options_init", "cd_screen", "cd_screen_ex", "cd_candidates", "cd_propagate",
                "cd_conjunctions_sort_device", "cd_conjunctions_free", "cd_candidates_free", "cd_status_str", "cd_last_error",
-               "cd_abi_version", "cd_kernel_launches", "cd_plan")
+               "cd_abi_version", "cd_kernel_launches", "cd_plan", "cd_shell_members")
 
 
 class CdError(RuntimeError):
@@ -84,7 +84,8 @@ class cd_options(C.Structure):
                 ("kepler_points", C.c_int), ("cell_factor", C.c_double),
                 ("batch_object_steps", C.c_size_t), ("round_steps", C.c_size_t),
                 ("profile_phases", C.c_int), ("l2_persist", C.c_int), ("grid_table", C.c_int),
-                ("stats", C.POINTER(cd_stats)), ("propagator", C.c_int)]
+                ("stats", C.POINTER(cd_stats)), ("propagator", C.c_int),
+                ("shell_lo", C.c_double), ("shell_hi", C.c_double)]
 
 
 class cd_plan_info(C.Structure):
@@ -134,6 +135,9 @@ def lib():
         L.cd_last_error.restype = C.c_char_p
         L.cd_abi_version.restype = C.c_int
         L.cd_kernel_launches.restype = C.c_uint64
+        L.cd_shell_members.restype = C.c_int
+        L.cd_shell_members.argtypes = [P(cd_elements), C.c_size_t, C.c_double, C.c_double, C.c_double,
+                                       C.c_void_p, P(C.c_size_t)]
         L.cd_plan.restype = C.c_int
         L.cd_plan.argtypes = [C.c_size_t, C.c_double, C.c_double, C.c_double, C.c_double, C.c_int,
                               C.c_size_t, P(cd_plan_info)]
@@ -199,6 +203,10 @@ def cd_kernel_launches() -> int:
     return int(lib().cd_kernel_launches())
 
 
+def cd_shell_members(el, n, lo, hi, gc, idx, count):
+    return lib().cd_shell_members(C.byref(el), n, lo, hi, gc, idx, C.byref(count))
+
+
 def cd_plan(n, t0, t1, dt, d, mode, mem_bytes, out):
     return lib().cd_plan(n, t0, t1, dt, d, mode, mem_bytes, C.byref(out))
 
@@ -227,7 +235,7 @@ class _Elements:
 def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None, stream=None,
                  cell_factor=None, batch_object_steps=None, round_steps=None,
                  outputs_on_device=False, inputs_on_device=False, profile_phases=False,
-                 l2_persist=None, grid_table=None, propagator=None):
+                 l2_persist=None, grid_table=None, propagator=None, shell=None):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -255,6 +263,8 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
         o.grid_table = int(grid_table)
     if propagator is not None:
         o.propagator = PROPAGATORS[propagator] if isinstance(propagator, str) else int(propagator)
+    if shell is not None:
+        o.shell_lo, o.shell_hi = float(shell[0]), float(shell[1])
     return o
 
 
@@ -339,3 +349,14 @@ def plan(n, t0, t1, dt, d, mode="grid", mem_bytes=0):
     out = cd_plan_info()
     _check(cd_plan(int(n), float(t0), float(t1), float(dt), float(d), _mode(mode), int(mem_bytes), out))
     return out.as_dict()
+
+
+def shell_members(pop, lo, hi, gc):
+    """Indices (uint32, increasing) of the objects a radial shard [lo, hi) must hold."""
+    E = _Elements(pop)
+    if E.on_device:
+        raise ValueError("shell_members takes host arrays")
+    idx = np.zeros(max(E.n, 1), dtype=np.uint32)
+    cnt = C.c_size_t()
+    _check(cd_shell_members(E.s, E.n, float(lo), float(hi), float(gc), idx.ctypes.data, cnt))
+    return idx[:cnt.value].copy()

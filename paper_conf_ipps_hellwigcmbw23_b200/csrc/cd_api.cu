@@ -431,6 +431,9 @@ cd_status validate_scalars(size_t n, double t0, double t1, double dt, double d, 
         return fail(CD_EINVAL, "need 0 <= rank < n_ranks");
     if (o.propagator != CD_PROP_KEPLER && o.propagator != CD_PROP_J2)
         return fail(CD_EINVAL, "unknown propagator %d", o.propagator);
+    if (!is_fin(o.shell_lo) || !is_fin(o.shell_hi) || o.shell_lo < 0.0 ||
+        (o.shell_hi != 0.0 && !(o.shell_hi > o.shell_lo)))
+        return fail(CD_EINVAL, "need shell_hi = 0 (no shard) or shell_hi > shell_lo >= 0");
     for (int c = 0; c < 3; ++c)
         if (!is_fin(o.grid_origin[c])) return fail(CD_EINVAL, "grid_origin must be finite");
     const double kk = std::floor((t1 - t0) / dt) + 1.0;
@@ -691,6 +694,8 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     g.reach = gc * (1.0 + 1e-9) + 1e-9;
     g.halfshell = L < 2.0 * gc ? 1 : 0;
     g.max_walk = (uint32_t)std::min<int64_t>(n + 1, 0xfffffffe);
+    g.band_lo2 = o.shell_hi > 0.0 ? o.shell_lo * o.shell_lo : 0.0;
+    g.band_hi2 = o.shell_hi > 0.0 ? o.shell_hi * o.shell_hi : HUGE_VAL;
     RefineParams P{t0, t1, dt, d, gc, nullptr};
 
     R.cand.st = st;
@@ -1159,6 +1164,8 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
         return fail(CD_EINVAL, "unknown mode %d", (int)mode);
     if (mode != CD_GRID && o.propagator != CD_PROP_KEPLER)
         return fail(CD_EINVAL, "CD_HYBRID and CD_LEGACY need CD_PROP_KEPLER (the filters assume fixed orbit planes)");
+    if (mode == CD_LEGACY && o.shell_hi != 0.0)
+        return fail(CD_EINVAL, "CD_LEGACY splits pairs by rank; radial shards apply to the grid");
     int64_t K = 0;
     TRY(validate_scalars(n, t0, t1, dt, d, o, &K));
     cd_stats stats;
@@ -1232,6 +1239,30 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
 }  // namespace
 
 extern "C" {
+
+cd_status cd_shell_members(const cd_elements* el, size_t n, double shell_lo, double shell_hi,
+                           double gc, uint32_t* idx, size_t* count)
+{
+    try {
+        if (!el || !el->a || !el->e || !idx || !count) return fail(CD_EINVAL, "NULL argument");
+        *count = 0;
+        if (!is_fin(shell_lo) || !is_fin(shell_hi) || !is_fin(gc) || shell_lo < 0.0 ||
+            !(shell_hi > shell_lo) || gc < 0.0)
+            return fail(CD_EINVAL, "need shell_hi > shell_lo >= 0 and g_c >= 0");
+        if (n >= 0xffffffffull) return fail(CD_EINVAL, "n too large");
+        size_t c = 0;
+        for (size_t i = 0; i < n; ++i) {
+            const double a = el->a[i], e = el->e[i];
+            if (!(a > 0.0) || !(e >= 0.0 && e < 1.0)) return fail(CD_EINVAL, "element %zu invalid", i);
+            // radius range [q, Q] meets [shell_lo, shell_hi + g_c)
+            if (a * (1.0 + e) >= shell_lo && a * (1.0 - e) < shell_hi + gc) idx[c++] = (uint32_t)i;
+        }
+        *count = c;
+        return CD_OK;
+    } catch (...) {
+        return fail(CD_EINTERNAL, "unexpected C++ exception");
+    }
+}
 
 void cd_options_init(cd_options* o)
 {

@@ -393,6 +393,9 @@ struct GridGeom {
     int halfshell;       // 1: own cell + 13 half-shell neighbours (L < 2 g_c); 0: the cells
                          // overlapping the ball |x - p| < g_c (L >= 2 g_c)
     uint32_t max_walk;   // list-walk bound (n): guards against a corrupted list
+    // radial shard (cd_options.shell_lo/hi): a candidate is kept iff the
+    // smaller of its two radii^2 lies in [band_lo2, band_hi2) (default [0, inf): all)
+    double band_lo2, band_hi2;
 };
 
 // Cell of position p: c = floor((p - o) / L) per axis (R7); frac = (p - o)/L - c in [0, 1).

@@ -293,6 +293,12 @@ __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_
 {
     const double dx = p[0] - ej.x, dy = p[1] - ej.y, dz = p[2] - ej.z;
     if (fma(dx, dx, fma(dy, dy, dz * dz)) < g.gc2) {
+        // radial shard: the pair belongs to the shard holding the smaller radius (identical
+        // positions on every shard, so exactly one shard keeps it)
+        const double ra = fma(p[0], p[0], fma(p[1], p[1], p[2] * p[2]));
+        const double rb = fma(ej.x, ej.x, fma(ej.y, ej.y, ej.z * ej.z));
+        const double rm = fmin(ra, rb);
+        if (!(rm >= g.band_lo2 && rm < g.band_hi2)) return;
         Cand cd;
         cd.i = r < j ? r : j;
         cd.j = r < j ? j : r;

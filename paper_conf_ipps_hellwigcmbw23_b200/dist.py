@@ -1,4 +1,5 @@
-"""Multi-GPU time slicing and the conjunction-list merge.
+"""Multi-GPU time slicing, radial object-space shards, and the conjunction-list merge
+(SURVEY.md 8(e), 8(f) row 2).
 
 One process per GPU.  The window's K sampling steps are split into contiguous slices; a call
 with ``rank=q, n_ranks=S`` screens steps [floor(q K / S), floor((q + 1) K / S)) and reports only
@@ -6,6 +7,15 @@ the minima it owns (owner rule), so slices partition the result set with no halo
 data-path collective.  The one real exchange is the final merge: an all-gather of the per-rank
 record counts, then of the (padded) 32-byte records, over NCCL / NVLink (``torch.distributed``
 is the plumbing), followed by the library's device sort by (i, j, step).
+
+Radial shards (SURVEY 8(f) row 2, for populations whose per-step grid would not fit one GPU;
+the paper names multiple GPUs for memory as future work): shard s of S keeps the
+candidates whose nearer-to-Earth partner is at radius |r| in [b_s, b_{s+1}) at t_k.  It holds
+only its members -- objects whose radius range [a(1-e), a(1+e)] meets [b_s, b_{s+1} + g_c): its
+own objects plus a g_c halo above the band -- so its grid and entries scale with n/S plus the
+halo and the eccentric objects that cross the band.  Positions are recomputed from the
+replicated elements on every shard (bit-identical), so the halo needs no exchange: a shard
+never reads another shard's grid.  Shards and time slices combine (rank = (shard, slice)).
 """
 from __future__ import annotations
 
@@ -74,3 +84,45 @@ def records_to_numpy(t):
     from . import CONJ_DTYPE
     a = t.cpu().numpy()
     return np.frombuffer(a.tobytes(), dtype=CONJ_DTYPE).copy()
+
+
+FAR_KM = 1.0e9   # upper bound of the outermost shard (cd_options.shell_hi must be finite)
+
+
+def shell_bounds(pop, S: int):
+    """S radial bands [b_s, b_{s+1}) with b_0 = 0, b_S = FAR_KM, balanced by the objects' mean
+    radius a (quantiles): each shard owns ~n/S objects."""
+    a = np.sort(np.asarray(pop["a"], dtype=np.float64))
+    inner = [float(a[min(len(a) - 1, (len(a) * s) // S)]) for s in range(1, S)]
+    return [0.0] + inner + [FAR_KM]
+
+
+def screen_shard(pop, t0, t1, dt, d, bounds, s, mode="grid", v_margin=7.8, **kw):
+    """Conjunctions of radial shard s (global object ids, sorted by (i, j, step)).  The member
+    subset keeps the global order, so the id map is monotonic and i < j survives it."""
+    from . import screen, shell_members, FIELDS
+    gc = d + v_margin * dt
+    lo, hi = bounds[s], bounds[s + 1]
+    idx = shell_members(pop, lo, hi, gc)
+    sub = {k: np.ascontiguousarray(np.asarray(pop[k])[idx]) for k in FIELDS}
+    if "propagator" in pop:
+        sub["propagator"] = pop["propagator"]
+    res = screen(sub, t0, t1, dt, d, mode=mode, v_margin=v_margin, shell=(lo, hi), **kw)
+    res["i"] = idx[res["i"]]
+    res["j"] = idx[res["j"]]
+    return res, len(idx)
+
+
+def candidates_shard(pop, t0, t1, dt, d, bounds, s, v_margin=7.8, **kw):
+    """The level-1 candidate set of radial shard s (global ids)."""
+    from . import candidates, shell_members, FIELDS
+    gc = d + v_margin * dt
+    lo, hi = bounds[s], bounds[s + 1]
+    idx = shell_members(pop, lo, hi, gc)
+    sub = {k: np.ascontiguousarray(np.asarray(pop[k])[idx]) for k in FIELDS}
+    if "propagator" in pop:
+        sub["propagator"] = pop["propagator"]
+    res = candidates(sub, t0, t1, dt, d, v_margin=v_margin, shell=(lo, hi), **kw)
+    res["i"] = idx[res["i"]]
+    res["j"] = idx[res["j"]]
+    return res

@@ -80,3 +80,82 @@ def test_slice_range_partitions():
             r = [cdist.slice_range(K, q, S) for q in range(S)]
             assert r[0][0] == 0 and r[-1][1] == K
             assert all(a[1] == b[0] for a, b in zip(r, r[1:]))
+
+
+# ----------------------------------------------------------------------------------------
+# radial object-space shards: host logic on CPU
+# ----------------------------------------------------------------------------------------
+
+def _shard_worker(rank, world, port, t1, d, ret):
+    """Each rank: its shard's members (the library's host helper cd_shell_members), the oracle's
+    candidate set on the member subset, the shard rule (smaller radius in the band) applied as
+    a plain definition, ids mapped back; gathered over gloo."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from tools import popgen
+        pop = popgen.random_population(1500, 21, "catalog", 300)
+        gc = oracle.cell_size(d, 1.0)
+        bounds = cdist.shell_bounds(pop, world)
+        lo, hi = bounds[rank], bounds[rank + 1]
+        import paper_conf_ipps_hellwigcmbw23_b200 as cds
+        idx = cds.shell_members(pop, lo, hi, gc)
+        sub = popgen.subset(pop, idx)
+        K = oracle.candidates_grid(sub, 0.0, t1, 1.0, gc)
+        keep = np.zeros(len(K), dtype=bool)
+        for q, c in enumerate(K):
+            x = oracle.propagate(popgen.subset(sub, [c["i"], c["j"]]), [float(c["step"])])[0]
+            rmin = np.min(np.linalg.norm(x, axis=1))
+            keep[q] = lo <= rmin < hi
+        K = K[keep]
+        K["i"], K["j"] = idx[K["i"]], idx[K["j"]]
+        rec = np.zeros((len(K), 32), dtype=np.uint8)
+        rec[:, :12] = np.frombuffer(K.tobytes(), dtype=np.uint8).reshape(-1, 12)
+        allrec = cdist.gather_records(torch.from_numpy(rec))
+        if rank == 0:
+            ret.put((allrec.numpy()[:, :12].tobytes(), len(idx)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_radial_shards_partition_candidates(orc, world):
+    from tools import popgen
+    t1, d = 40.0, 20.0
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_shard_worker, args=(r, world, port, t1, d, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    data, nmem = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=300)
+        assert p.exitcode == 0
+    got = np.sort(np.frombuffer(data, dtype=orc.CAND_DTYPE), order=["i", "j", "step"])
+    pop = popgen.random_population(1500, 21, "catalog", 300)
+    whole = orc.candidates_grid(pop, 0.0, t1, 1.0, orc.cell_size(d, 1.0))
+    assert len(whole) > 50
+    assert np.array_equal(got, whole)     # disjoint shards, union = the unsharded set
+    assert nmem < 1500                    # rank 0 holds a strict subset
+
+
+def test_shell_bounds_and_members():
+    import paper_conf_ipps_hellwigcmbw23_b200 as cds
+    from tools import popgen
+    pop = popgen.random_population(5000, 22, "catalog", 1000)
+    for S in (1, 2, 4, 8):
+        b = cdist.shell_bounds(pop, S)
+        assert len(b) == S + 1 and b[0] == 0.0 and all(x < y for x, y in zip(b, b[1:]))
+        own = np.histogram(pop["a"], bins=b)[0]
+        assert own.max() <= 5000 // S + 2            # balanced by mean radius
+        gc = 9.8
+        for s in range(S):
+            idx = cds.shell_members(pop, b[s], b[s + 1], gc)
+            q, Q = pop["a"] * (1 - pop["e"]), pop["a"] * (1 + pop["e"])
+            want = np.where((Q >= b[s]) & (q < b[s + 1] + gc))[0]
+            assert np.array_equal(idx, want.astype(np.uint32))
+    with pytest.raises(cds.CdError):
+        cds.shell_members(pop, 7000.0, 7000.0, 1.0)
