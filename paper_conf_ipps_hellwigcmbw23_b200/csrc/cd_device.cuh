@@ -251,6 +251,19 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
             den += ia * fma(ct, rea, st * ima) + ib * fma(-ct, reb, st * imb);
         }
         delta = rho * (num * rcp_fast(den));
+        // the root lies inside the contour, |E - c| < rho: a non-finite or out-of-range quotient
+        // (rounding next to a degenerate node) falls back to Newton from the contour centre
+        if (!(fabs(delta) <= rho)) {
+            double x = c;
+            for (int it = 0; it < 12; ++it) {
+                double sx, cx;
+                sincos_fast(x, sx, cx);
+                const double dx = (x - e * sx - M) / fma(-e, cx, 1.0);
+                x -= dx;
+                if (fabs(dx) <= 1e-16 * fmax(1.0, fabs(x))) break;
+            }
+            delta = fmin(fmax(x - c, -rho), rho);
+        }
     }
     E = c + delta;
     double sd, cd;
