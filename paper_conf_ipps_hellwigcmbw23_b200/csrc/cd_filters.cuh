@@ -43,47 +43,58 @@ __device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o)
     o.pad = 0.0;
 }
 
-// mean anomaly of true anomaly f, in [-pi, pi]: f is reduced to [-pi, pi] first so the half-angle
-// formula stays on its principal branch (window ends on different branches would cancel a window)
-__device__ __forceinline__ double mean_of_true(double f, double e)
+// Node geometry of one orbit of a pair (reading R17), all algebraic: the mutual node line is a
+// unit vector in the orbit plane, so its components along P and Q are the cosine and sine of its
+// true anomaly f; the window half-angle a = asin(s) has sin a = s, cos a = sqrt(1 - s^2).  The
+// opposite node (f + pi) flips the sign of (cos f, sin f).
+struct NodeGeom {
+    double cf, sf;   // cos f, sin f of the ascending mutual node
+    double sa, ca;   // sin a, cos a of the window half-angle
+};
+
+// Mean anomaly of the true anomaly with cosine c and sine s, in [-pi, pi] (principal branch):
+//   sin E = sqrt(1 - e^2) s / (1 + e c),  cos E = (e + c) / (1 + e c),  M = E - e sin E
+__device__ __forceinline__ double mean_of_true_cs(double c, double s, double e)
 {
-    f = remainder(f, kTwoPiH);
-    double sf, cf;
-    sincos(0.5 * f, &sf, &cf);
-    const double E = 2.0 * atan2(sqrt(1.0 - e) * sf, sqrt(1.0 + e) * cf);
-    return E - e * sin(E);
+    const double w = sqrt((1.0 - e) * (1.0 + e));
+    const double E = atan2(w * s, e + c);
+    return E - e * (w * s / fma(e, c, 1.0));
 }
 
-// radius range over true anomalies [f1, f2], f2 - f1 < pi
-__device__ __forceinline__ void radius_range(const HOrbit& o, double f1, double f2, double& rmin,
-                                             double& rmax)
+// radius range over the true anomalies (f - a, f + a) of node `sg` (+1: f, -1: f + pi), a < pi/2:
+// the ends r = p / (1 + e cos(f -+ a)), widened to the perigee radius if the interval contains
+// f = 0 (cos f >= cos a) and to the apogee radius if it contains f = pi (-cos f >= cos a)
+__device__ __forceinline__ void radius_range(const HOrbit& o, const NodeGeom& g, double sg,
+                                             double& rmin, double& rmax)
 {
-    const double r1 = o.p / (1.0 + o.e * cos(f1)), r2 = o.p / (1.0 + o.e * cos(f2));
+    const double cf = sg * g.cf, sf = sg * g.sf;
+    const double c1 = fma(cf, g.ca, sf * g.sa), c2 = fma(cf, g.ca, -sf * g.sa);
+    const double r1 = o.p / fma(o.e, c1, 1.0), r2 = o.p / fma(o.e, c2, 1.0);
     rmin = fmin(r1, r2);
     rmax = fmax(r1, r2);
-    if (ceil(f1 / kTwoPiH) * kTwoPiH <= f2) rmin = o.q;                  // perigee inside
-    if (kPiH + ceil((f1 - kPiH) / kTwoPiH) * kTwoPiH <= f2) rmax = o.Q;  // apogee inside
+    if (cf >= g.ca) rmin = o.q;    // perigee inside
+    if (-cf >= g.ca) rmax = o.Q;   // apogee inside
 }
 
-// first-occurrence time window [tl, th] (mod T) of true anomaly in (fc - al, fc + al)
-__device__ __forceinline__ void node_window(const HOrbit& o, double fc, double al, double& tl,
-                                            double& th)
+// first-occurrence time window [tl, th] (mod T) of the true anomaly in (f - a, f + a) of node sg
+__device__ __forceinline__ void node_window(const HOrbit& o, const NodeGeom& g, double sg,
+                                            double& tl, double& th)
 {
-    const double Ml = mean_of_true(fc - al, o.e);
-    double Mh = mean_of_true(fc + al, o.e);
+    const double cf = sg * g.cf, sf = sg * g.sf;
+    const double Ml = mean_of_true_cs(fma(cf, g.ca, sf * g.sa), fma(sf, g.ca, -cf * g.sa), o.e);
+    double Mh = mean_of_true_cs(fma(cf, g.ca, -sf * g.sa), fma(sf, g.ca, cf * g.sa), o.e);
     if (Mh < Ml) Mh += kTwoPiH;
     tl = (Ml - o.M0) / o.nm;
     th = (Mh - o.M0) / o.nm;
 }
 
 // Pair geometry of the filter chain (reading R17).  Returns 1 if the apogee/perigee filter
-// rejects the pair; otherwise 0 with coplanar set, and for non-coplanar pairs the node-window
-// half-angles aA, aB and the true anomalies fA, fB of the mutual node line in each orbit.
+// rejects the pair; otherwise 0 with coplanar set, and for non-coplanar pairs the node geometry
+// of each orbit.
 //   AP:        exclude iff max(q_A, q_B) - min(Q_A, Q_B) > d
 //   coplanar:  s_X = d / (q_X sin D) >= 1 for A or B, or q_A cos(asin s_A) + q_B cos(asin s_B) <= d
 __device__ __forceinline__ int pair_geometry(const HOrbit& A, const HOrbit& B, double d,
-                                             bool& coplanar, double& aA, double& aB, double& fA,
-                                             double& fB)
+                                             bool& coplanar, NodeGeom& gA, NodeGeom& gB)
 {
     if (fmax(A.q, B.q) - fmin(A.Q, B.Q) > d) return 1;
     const double c[3] = {A.h[1] * B.h[2] - A.h[2] * B.h[1], A.h[2] * B.h[0] - A.h[0] * B.h[2],
@@ -92,29 +103,35 @@ __device__ __forceinline__ int pair_geometry(const HOrbit& A, const HOrbit& B, d
     const double sA = sD > 0.0 ? d / (A.q * sD) : 2.0;
     const double sB = sD > 0.0 ? d / (B.q * sD) : 2.0;
     coplanar = sA >= 1.0 || sB >= 1.0;
-    aA = aB = fA = fB = 0.0;
-    if (!coplanar) {
-        aA = asin(sA);
-        aB = asin(sB);
-        coplanar = A.q * cos(aA) + B.q * cos(aB) <= d;
-    }
+    if (coplanar) return 0;
+    gA.sa = sA;
+    gB.sa = sB;
+    gA.ca = sqrt((1.0 - sA) * (1.0 + sA));
+    gB.ca = sqrt((1.0 - sB) * (1.0 + sB));
+    coplanar = A.q * gA.ca + B.q * gB.ca <= d;
     if (coplanar) return 0;
     const double nn[3] = {c[0] / sD, c[1] / sD, c[2] / sD};
-    fA = atan2(nn[0] * A.Qv[0] + nn[1] * A.Qv[1] + nn[2] * A.Qv[2],
-               nn[0] * A.P[0] + nn[1] * A.P[1] + nn[2] * A.P[2]);
-    fB = atan2(nn[0] * B.Qv[0] + nn[1] * B.Qv[1] + nn[2] * B.Qv[2],
-               nn[0] * B.P[0] + nn[1] * B.P[1] + nn[2] * B.P[2]);
+    double x = nn[0] * A.P[0] + nn[1] * A.P[1] + nn[2] * A.P[2];
+    double y = nn[0] * A.Qv[0] + nn[1] * A.Qv[1] + nn[2] * A.Qv[2];
+    double k = 1.0 / sqrt(x * x + y * y);
+    gA.cf = x * k;
+    gA.sf = y * k;
+    x = nn[0] * B.P[0] + nn[1] * B.P[1] + nn[2] * B.P[2];
+    y = nn[0] * B.Qv[0] + nn[1] * B.Qv[1] + nn[2] * B.Qv[2];
+    k = 1.0 / sqrt(x * x + y * y);
+    gB.cf = x * k;
+    gB.sf = y * k;
     return 0;
 }
 
-// orbit-path filter at one mutual node (off = 0 or pi): true iff the radial ranges of A and B
-// over their node windows are more than d apart (|r_A - r_B| >= ||r_A| - |r_B||)
-__device__ __forceinline__ bool node_closed(const HOrbit& A, const HOrbit& B, double d, double fA,
-                                            double fB, double aA, double aB, double off)
+// orbit-path filter at node sg (+1 / -1): true iff the radial ranges of A and B over their node
+// windows are more than d apart (|r_A - r_B| >= ||r_A| - |r_B||)
+__device__ __forceinline__ bool node_closed(const HOrbit& A, const HOrbit& B, double d,
+                                            const NodeGeom& gA, const NodeGeom& gB, double sg)
 {
     double rAl, rAh, rBl, rBh;
-    radius_range(A, fA + off - aA, fA + off + aA, rAl, rAh);
-    radius_range(B, fB + off - aB, fB + off + aB, rBl, rBh);
+    radius_range(A, gA, sg, rAl, rAh);
+    radius_range(B, gB, sg, rBl, rBh);
     return fmax(rAl, rBl) - fmin(rAh, rBh) > d;
 }
 

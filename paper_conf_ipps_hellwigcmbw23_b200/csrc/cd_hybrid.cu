@@ -74,8 +74,8 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
         const HOrbit A = hr[cd.i], B = hr[cd.j];
         const double d = P.d;
         bool coplanar;
-        double aA, aB, fA, fB;
-        if (pair_geometry(A, B, d, coplanar, aA, aB, fA, fB)) {   // apogee / perigee
+        NodeGeom gA, gB;
+        if (pair_geometry(A, B, d, coplanar, gA, gB)) {   // apogee / perigee
             count1(&ctrl->n_ap);
             continue;
         }
@@ -90,12 +90,12 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
         bool any_node = false;
         int nwin = 0;
         for (int node = 0; node < 2; ++node) {
-            const double off = node ? kPiH : 0.0;
-            if (node_closed(A, B, d, fA, fB, aA, aB, off)) continue;   // orbit path: node closed
+            const double sg = node ? -1.0 : 1.0;   // mutual node / opposite node (f + pi)
+            if (node_closed(A, B, d, gA, gB, sg)) continue;   // orbit path: node closed
             any_node = true;
             double atl, ath, btl, bth;
-            node_window(A, fA + off, aA, atl, ath);
-            node_window(B, fB + off, aB, btl, bth);
+            node_window(A, gA, sg, atl, ath);
+            node_window(B, gB, sg, btl, bth);
             double wa[4], wb[4];
             const int na = window_copies(atl - tk, ath - tk, kTwoPiH / A.nm, lo, hi, wa);
             const int nb = window_copies(btl - tk, bth - tk, kTwoPiH / B.nm, lo, hi, wb);
@@ -113,8 +113,8 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
                 }
         }
 #ifdef CD_DEBUG_FILTER
-        printf("filter i=%u j=%u k=%u aA=%.17g aB=%.17g fA=%.17g fB=%.17g lo=%g hi=%g any=%d nwin=%d A.M0=%.17g A.nm=%.17g B.M0=%.17g B.nm=%.17g\n",
-               cd.i, cd.j, cd.step, aA, aB, fA, fB, lo, hi, (int)any_node, nwin, A.M0, A.nm, B.M0, B.nm);
+        printf("filter i=%u j=%u k=%u lo=%g hi=%g any=%d nwin=%d\n", cd.i, cd.j, cd.step, lo, hi,
+               (int)any_node, nwin);
 #endif
         if (!any_node) count1(&ctrl->n_path);
         else if (nwin == 0) count1(&ctrl->n_time);

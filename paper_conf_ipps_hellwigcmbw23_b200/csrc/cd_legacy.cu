@@ -88,8 +88,8 @@ __global__ void __launch_bounds__(256) k_legacy_filter(LegacyParams P, const HOr
         }
         const HOrbit A = hr[i], B = hr[j];
         bool coplanar;
-        double aA, aB, fA, fB;
-        pair_geometry(A, B, d, coplanar, aA, aB, fA, fB);
+        NodeGeom gA, gB;
+        pair_geometry(A, B, d, coplanar, gA, gB);
         if (coplanar) {
             count1(&ctrl->n_coplanar);
             emit_interval(i, j, 4u /* CD_FLAG_COPLANAR */, P.t0, P.t1, P, w, wcap, n_work);
@@ -99,12 +99,12 @@ __global__ void __launch_bounds__(256) k_legacy_filter(LegacyParams P, const HOr
         int nint = 0;
         const double TA = kTwoPiH / A.nm, TB = kTwoPiH / B.nm;
         for (int node = 0; node < 2; ++node) {
-            const double off = node ? kPiH : 0.0;
-            if (node_closed(A, B, d, fA, fB, aA, aB, off)) continue;   // orbit path
+            const double sg = node ? -1.0 : 1.0;   // mutual node / opposite node (f + pi)
+            if (node_closed(A, B, d, gA, gB, sg)) continue;   // orbit path
             any_node = true;
             double atl, ath, btl, bth;
-            node_window(A, fA + off, aA, atl, ath);
-            node_window(B, fB + off, aB, btl, bth);
+            node_window(A, gA, sg, atl, ath);
+            node_window(B, gB, sg, btl, bth);
             // every window copy k of each object overlapping [t0, t1], merged in time order
             double ka = floor((P.t0 - ath) / TA), kb = floor((P.t0 - bth) / TB);
             for (int guard = 0; guard < (1 << 22); ++guard) {
