@@ -119,7 +119,7 @@ typedef struct {
     uint64_t object_steps;     /* n * steps                                                    */
     uint64_t candidates;       /* |K| for this slice (hybrid: coarse candidates)              */
     uint64_t refined;          /* candidates that survived the conservative linear pre-filter
-                                  (hybrid: non-coplanar time-window work items + coplanar)    */
+                                  (hybrid: time-window work items + coplanar candidates)     */
     uint64_t conjunctions;     /* reported rows                                               */
     uint64_t hybrid_ap_rejected, hybrid_coplanar, hybrid_path_rejected, hybrid_time_rejected;
     uint64_t kernel_launches;  /* CUDA kernels launched by this call                          */

@@ -11,12 +11,14 @@ The same names as the C ABI are exported (``cd_screen``, ``cd_screen_ex``, ``cd_
 from __future__ import annotations
 
 import ctypes as C
+import os
 from pathlib import Path
 
 import numpy as np
 
 PKG = Path(__file__).resolve().parent
-LIB_PATH = PKG / "libcdscreen.so"
+# CDSCREEN_LIB: load an alternative build of the same library (A/B timing of kernel variants)
+LIB_PATH = Path(os.environ.get("CDSCREEN_LIB", str(PKG / "libcdscreen.so")))
 
 CD_OK, CD_EINVAL, CD_ENOMEM, CD_ECUDA, CD_ENCCL, CD_ERANGE, CD_EINTERNAL, CD_ENODEV = range(8)
 CD_GRID, CD_HYBRID, CD_LEGACY = 0, 1, 2

@@ -27,29 +27,6 @@ namespace cdh {
 
 using namespace filt;
 
-namespace {
-
-// the (at most one per period) copy of the periodic window [tl, th] + k T overlapping [lo, hi];
-// windows are shorter than half a period and [lo, hi] (one coarse cell) is far shorter than a
-// period, so at most two copies can touch it
-__device__ __forceinline__ int window_copies(double tl, double th, double T, double lo, double hi,
-                                             double out[4])
-{
-    int c = 0;
-    const double k0 = floor((lo - th) / T);
-    for (int q = 0; q < 3; ++q) {
-        const double a = tl + (k0 + q) * T, b = th + (k0 + q) * T;
-        if (b < lo || a > hi) continue;
-        if (c < 2) {
-            out[2 * c] = fmax(a, lo);
-            out[2 * c + 1] = fmin(b, hi);
-            ++c;
-        }
-    }
-    return c;
-}
-
-}  // namespace
 
 __global__ void k_build_hrec(Orbits O, HOrbit* __restrict__ hr)
 {
@@ -60,7 +37,10 @@ __global__ void k_build_hrec(Orbits O, HOrbit* __restrict__ hr)
     hr[r] = o;
 }
 
-__global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P, const Cand* __restrict__ q,
+#ifndef CD_FILTER_MINB
+#define CD_FILTER_MINB 1
+#endif
+__global__ void __launch_bounds__(256, CD_FILTER_MINB) k_hybrid_filter(Orbits O, RefineParams P, const Cand* __restrict__ q,
                                                        size_t qcap, Work* __restrict__ w, size_t wcap,
                                                        unsigned long long* n_work,
                                                        Conj* __restrict__ out, size_t ocap, Ctrl* ctrl)
@@ -71,17 +51,26 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
     const size_t stride = (size_t)gridDim.x * blockDim.x;
     for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < nc; idx += stride) {
         const Cand cd = q[idx];
-        const HOrbit A = hr[cd.i], B = hr[cd.j];
         const double d = P.d;
+        // apogee / perigee first, from 16 bytes of each record
+        if (fmax(hr[cd.i].q, hr[cd.j].q) - fmin(hr[cd.i].Q, hr[cd.j].Q) > d) {
+            count1(&ctrl->n_ap);
+            continue;
+        }
+        const HOrbit A = hr[cd.i], B = hr[cd.j];
         bool coplanar;
         NodeGeom gA, gB;
         if (pair_geometry(A, B, d, coplanar, gA, gB)) {   // apogee / perigee
             count1(&ctrl->n_ap);
             continue;
         }
-        if (coplanar) {   // same procedure as the grid-based variant
+        if (coplanar) {   // same procedure as the grid-based variant (set-up in k_brent)
             count1(&ctrl->n_coplanar);
-            grid_refine_item(O, P, cd, 4u /* CD_FLAG_COPLANAR */, w, wcap, n_work, out, ocap, ctrl);
+            Work it;
+            it.i = cd.i; it.j = cd.j; it.step = cd.step;
+            it.flags = 4u /* CD_FLAG_COPLANAR */ | kWorkSetup;
+            it.lo = it.hi = 0.0;
+            append(w, wcap, n_work, it);
             continue;
         }
         // owner cell of the coarse step, relative to t_k
@@ -96,12 +85,18 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
             double atl, ath, btl, bth;
             node_window(A, gA, sg, atl, ath);
             node_window(B, gB, sg, btl, bth);
-            double wa[4], wb[4];
-            const int na = window_copies(atl - tk, ath - tk, kTwoPiH / A.nm, lo, hi, wa);
-            const int nb = window_copies(btl - tk, bth - tk, kTwoPiH / B.nm, lo, hi, wb);
-            for (int x = 0; x < na; ++x)
-                for (int y = 0; y < nb; ++y) {
-                    const double l = fmax(wa[2 * x], wb[2 * y]), h = fmin(wa[2 * x + 1], wb[2 * y + 1]);
+            // the copies k T of each periodic window that meet the owner cell [lo, hi] (windows
+            // are shorter than half a period and the cell far shorter than a period: at most two
+            // of three consecutive copies), intersected pairwise
+            const double TA = kTwoPiH / A.nm, TB = kTwoPiH / B.nm;
+            const double ka = floor((lo - (ath - tk)) / TA), kb = floor((lo - (bth - tk)) / TB);
+            for (int x = 0; x < 3; ++x) {
+                const double al = fmax(atl - tk + (ka + x) * TA, lo), ah = fmin(ath - tk + (ka + x) * TA, hi);
+                if (!(ah >= al)) continue;
+                for (int y = 0; y < 3; ++y) {
+                    const double bl = fmax(btl - tk + (kb + y) * TB, lo), bh = fmin(bth - tk + (kb + y) * TB, hi);
+                    if (!(bh >= bl)) continue;
+                    const double l = fmax(al, bl), h = fmin(ah, bh);
                     if (h > l) {
                         Work it;
                         it.i = cd.i; it.j = cd.j; it.step = cd.step; it.flags = 0u;
@@ -111,6 +106,7 @@ __global__ void __launch_bounds__(256) k_hybrid_filter(Orbits O, RefineParams P,
                         ++nwin;
                     }
                 }
+            }
         }
 #ifdef CD_DEBUG_FILTER
         printf("filter i=%u j=%u k=%u lo=%g hi=%g any=%d nwin=%d\n", cd.i, cd.j, cd.step, lo, hi,

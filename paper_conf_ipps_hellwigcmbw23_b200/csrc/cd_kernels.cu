@@ -647,7 +647,13 @@ __global__ void __launch_bounds__(128) k_brent(Orbits O, RefineParams P, const W
     if (nw > wcap) nw = wcap;
     const size_t stride = (size_t)gridDim.x * blockDim.x;
     for (size_t idx = blockIdx.x * (size_t)blockDim.x + threadIdx.x; idx < nw; idx += stride) {
-        const Work it = w[idx];
+        Work it = w[idx];
+        if (it.flags & kWorkSetup) {   // hybrid coplanar candidate: grid-variant set-up here
+            it.flags &= ~kWorkSetup;
+            Cand cd;
+            cd.i = it.i; cd.j = it.j; cd.step = it.step;
+            if (!grid_refine_setup(O, P, cd, it.flags, it.lo, it.hi, out, ocap, ctrl)) continue;
+        }
         const double tk = fma((double)it.step, P.dt, P.t0);
         double x, fx;
         if (!brent_min(O, it.i, it.j, tk, it.lo, it.hi, x, fx)) continue;
