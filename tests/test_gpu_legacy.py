@@ -111,3 +111,14 @@ def test_legacy_errors():
         cds.candidates(pop, 0.0, 90.0, 1.0, 2.0, mode="legacy")
     assert ei.value.status == cds.CD_EINVAL
     assert len(cds.screen(popgen.subset(pop, [3]), 0.0, 90.0, 1.0, 2.0, mode="legacy")) == 0
+
+
+def test_legacy_config2_full_window():
+    """BASELINE config 2 at full size (30,000 objects, the whole 24 h at 1 s): the legacy chain on
+    the device against oracle O5 element by element, and the filter-stage counts."""
+    pop, cfg, _ = popgen.make_config(2)
+    Lg, st = cds.screen(pop, cfg.t0, cfg.t1, cfg.dt_grid, cfg.d, mode="legacy", return_stats=True)
+    Lo, cnt = oracle.legacy(pop, cfg.t0, cfg.t1, cfg.dt_grid, cfg.d)
+    _check_counts(st, cnt)
+    res = parity.compare_legacy(pop, Lg, Lo, cfg.t0, cfg.t1, cfg.dt_grid, cfg.d)
+    assert res["matched"] > 7000

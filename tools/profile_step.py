@@ -25,7 +25,7 @@ def main():
     import paper_conf_ipps_hellwigcmbw23_b200 as cds
     from tools import popgen
     pop, cfg, _ = popgen.make_config(args.config, n=args.n)
-    dt = cfg.dt_grid if args.variant == "grid" else cfg.dt_hybrid
+    dt = cfg.dt_hybrid if args.variant == "hybrid" else (cfg.dt_grid or 1.0)
     dpop = {k: torch.from_numpy(v).cuda() for k, v in pop.items()}
     kw = {}
     if args.cell_factor is not None:
