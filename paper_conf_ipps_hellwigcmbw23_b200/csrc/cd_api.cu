@@ -693,6 +693,8 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     g.gc2 = gc * gc;
     g.reach = gc * (1.0 + 1e-9) + 1e-9;
     g.halfshell = L < 2.0 * gc ? 1 : 0;
+    // block-level candidate staging pays at dense candidate rates (>= 0.05 per object-step)
+    g.stage = est_step / std::max<double>(1.0, (double)n) >= 0.05 ? 1 : 0;
     g.max_walk = (uint32_t)std::min<int64_t>(n + 1, 0xfffffffe);
     g.band_lo2 = o.shell_hi > 0.0 ? o.shell_lo * o.shell_lo : 0.0;
     g.band_hi2 = o.shell_hi > 0.0 ? o.shell_hi * o.shell_hi : HUGE_VAL;
@@ -1041,7 +1043,9 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             ocap = ncap;
         }
         if (!settled) {   // first round done: pick the cell edge from the measured density
-            const double m = choose_cell_factor((double)hctrl->n_cand / ((double)rd.Rk * (double)n));
+            const double dens = (double)hctrl->n_cand / ((double)rd.Rk * (double)n);
+            const double m = choose_cell_factor(dens);
+            g.stage = dens >= 0.05 ? 1 : 0;
             L = gc * m;
             if (L < gc * (1.0 + 1e-12)) L = gc * (1.0 + 1e-12);
             g.inv_cell = 1.0 / L;

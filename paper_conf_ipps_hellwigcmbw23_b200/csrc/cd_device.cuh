@@ -409,6 +409,7 @@ struct GridGeom {
     // radial shard (cd_options.shell_lo/hi): a candidate is kept iff the
     // smaller of its two radii^2 lies in [band_lo2, band_hi2) (default [0, inf): all)
     double band_lo2, band_hi2;
+    int stage;           // 1: stage candidates per block in shared memory (dense candidate rates)
 };
 
 // Cell of position p: c = floor((p - o) / L) per axis (R7); frac = (p - o)/L - c in [0, 1).
