@@ -23,17 +23,18 @@ static inline unsigned blocks_for(int64_t n, int t) { return (unsigned)((n + t -
 // With pdl, the launch may begin while the previous kernel in the stream is still running
 // (programmatic dependent launch); the kernel orders its dependent part with griddepcontrol.wait.
 template <typename... KArgs, typename... Args>
-static cudaError_t launch_ex(void (*kern)(KArgs...), dim3 grid, dim3 block, cudaStream_t st,
-                             const L2Win* win, bool pdl, Args... args)
+static cudaError_t launch_ex(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                             cudaStream_t st, const L2Win* win, bool pdl, Args... args)
 {
     const bool w = win && win->on;
     if (!w && !pdl) {
-        kern<<<grid, block, 0, st>>>(args...);
+        kern<<<grid, block, smem, st>>>(args...);
         return cudaGetLastError();
     }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = grid;
     cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
     cfg.stream = st;
     cudaLaunchAttribute at[2];
     unsigned na = 0;
@@ -293,8 +294,10 @@ __constant__ int8_t kHalfShell[14][3] = {
 // A dense coarse grid (the hybrid's 1.4 candidates per object-step) otherwise serialises on the
 // queue counter (hybrid k_step 556 -> 284 us per 1M-object step); a sparse one (the grid
 // variant's 0.004) does not need it and skips the block barriers (64 vs 68 us).
+// The buffer is dynamic shared memory, requested only for staged launches: a sparse step keeps
+// the whole L1 (static shared memory here cost the grid variant 3 %).
 constexpr unsigned kSCand = 1024;
-__shared__ Cand s_cand[kSCand];
+extern __shared__ Cand s_cand[];
 __shared__ unsigned s_ncand;
 __shared__ unsigned long long s_cbase;
 
@@ -638,13 +641,15 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
     const int64_t blocks = a.build_B * (a.nbA + a.nbB) + a.nCblocks;
     if (blocks == 0) return cudaSuccess;
     lc.bump();
+    const size_t smem = a.g.stage ? sizeof(Cand) * kSCand : 0;   // candidate staging buffer
     if (a.O.j2) {   // J2 secular propagator: the rotation is compiled into its own instances
         if (a.chained)
-            return launch_ex(k_step<true, 1>, dim3((unsigned)blocks), dim3(256), st, win, a.pdl != 0, a);
-        return launch_ex(k_step<false, 1>, dim3((unsigned)blocks), dim3(256), st, win, false, a);
+            return launch_ex(k_step<true, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, a.pdl != 0, a);
+        return launch_ex(k_step<false, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
     }
-    if (a.chained) return launch_ex(k_step<true, 0>, dim3((unsigned)blocks), dim3(256), st, win, a.pdl != 0, a);
-    return launch_ex(k_step<false, 0>, dim3((unsigned)blocks), dim3(256), st, win, false, a);
+    if (a.chained)
+        return launch_ex(k_step<true, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, a.pdl != 0, a);
+    return launch_ex(k_step<false, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
 }
 
 // ---------------------------------------------------------------------------------------
