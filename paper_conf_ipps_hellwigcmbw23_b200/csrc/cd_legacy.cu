@@ -15,7 +15,9 @@
 //                    [t_k - dt/2, t_k + dt/2) meets the interval is a sample; with
 //                    v_max = v_p,A + v_p,B (perigee speeds, >= |v_A - v_B| always), a minimum
 //                    below d within dt/2 of t_k has D(t_k) < d + v_max dt/2, so only such samples
-//                    run Brent on [t_k - dt, t_k + dt] n [lo, hi] (cd_refine.cuh); a minimum is
+//                    run Brent on [t_k - dt, t_k + dt] n [lo, hi] (cd_refine.cuh), and a sample at
+//                    distance D skips the (D - gate)/(v_max dt) steps that cannot reach the gate
+//                    (long coplanar searches: pairs far apart are skipped in strides); a minimum is
 //                    reported by its owner step (reading R9), with D < d and TCA in [t0, t1].
 //                    Degenerate pairs (|v_A - v_B| < 1e-9 km/s: no isolated minimum) are skipped.
 #include "cd_filters.cuh"
@@ -148,10 +150,21 @@ __global__ void __launch_bounds__(128) k_legacy_search(Orbits O, LegacyParams P,
         const double vmax = sqrt(kMu * (1.0 + A.e) / A.q) + sqrt(kMu * (1.0 + B.e) / B.q);
         const double gate = P.d + vmax * 0.5 * P.dt + 1e-9;
         const double gate2 = gate * gate;
-        for (uint32_t s = lane; s < cnt; s += 32) {
+        // each lane walks a contiguous sub-span; a sample far outside the gate skips the steps
+        // that cannot be gated: |dD/dt| <= v_max, so D >= D_k - v_max m dt >= gate for the next
+        // m = floor((D_k - gate) / (v_max dt)) steps
+        const uint32_t per = (cnt + 31) / 32;
+        const uint32_t s_end = min(cnt, (lane + 1) * per);
+        const double inv_step = 1.0 / (vmax * P.dt);
+        for (uint32_t s = lane * per; s < s_end; ++s) {
             const uint32_t k = it.step + s;
             const double tk = fma((double)k, P.dt, P.t0);
-            if (!(dist2_at(O, it.i, it.j, tk) < gate2)) continue;
+            const double D2 = dist2_at(O, it.i, it.j, tk);
+            if (!(D2 < gate2)) {
+                const double m = floor((sqrt(D2) - gate) * inv_step);
+                if (m >= 1.0) s += (uint32_t)fmin(m, (double)per);
+                continue;
+            }
             double ri[3], vi[3], rj[3], vj[3];
             state<true>(O, it.i, tk, ri, vi);
             state<true>(O, it.j, tk, rj, vj);
