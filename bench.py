@@ -197,13 +197,17 @@ def run_ours(args):
         if world > 1:
             dist.barrier()
 
+    # device scratch memory from PyTorch's caching allocator on the bench stream (cd_options.alloc)
+    talloc = cds.TorchAllocator(dev.index, stream.cuda_stream) if args.torch_alloc else None
+
     def one_step(s, profile, host_inputs=False):
         q = (s * world + rank) % S
         E = cds._Elements(pop if host_inputs else dpop)
         st = cds.cd_stats()
         opt = cds.make_options(rank=q, n_ranks=S, device=dev.index, stream=stream.cuda_stream,
                                inputs_on_device=not host_inputs,
-                               outputs_on_device=not host_inputs, profile_phases=profile)
+                               outputs_on_device=not host_inputs, profile_phases=profile,
+                               allocator=talloc)
         import ctypes as C
         opt.stats = C.pointer(st)
         out = cds.cd_conjunctions()
@@ -281,7 +285,7 @@ def run_ours(args):
             E = cds._Elements(dpop)
             st = cds.cd_stats()
             opt = cds.make_options(rank=q, n_ranks=S, device=dev.index, stream=stream.cuda_stream,
-                                   inputs_on_device=True, outputs_on_device=True)
+                                   inputs_on_device=True, outputs_on_device=True, allocator=talloc)
             import ctypes as C
             opt.stats = C.pointer(st)
             out = cds.cd_conjunctions()
@@ -331,7 +335,7 @@ def run_ours(args):
         e0.record(stream)
         q = (s * world + rank) % S
         recs = cds.screen(pin_np, cfg.t0, cfg.t1, dt, cfg.d, mode=args.variant, rank=q, n_ranks=S,
-                          device=dev.index, stream=stream.cuda_stream)
+                          device=dev.index, stream=stream.cuda_stream, allocator=talloc)
         e1.record(stream)
         torch.cuda.synchronize()
         e2e_ms.append(e0.elapsed_time(e1))
@@ -394,6 +398,8 @@ def run_ours(args):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": dict(workload_config(args, cfg, n, dt, K),
                            slices=S, wall_s_window=tot_ms / 1e3 * (S / (args.steps * world)),
+                           device_memory="PyTorch caching allocator (cd_options.alloc)" if args.torch_alloc
+                           else "library stream-ordered pool",
                            conjunctions=nconj, parallelism=f"time-slice x{world}"),
             "step_ms": {"min": float(np.min(times)), "median": float(np.median(times)),
                         "max": float(np.max(times))},
@@ -432,6 +438,8 @@ def main():
     ap.add_argument("--cpu-steps", type=int, default=128)
     ap.add_argument("--ref-steps", type=int, default=None)
     ap.add_argument("--e2e-steps", type=int, default=None)
+    ap.add_argument("--no-torch-alloc", dest="torch_alloc", action="store_false",
+                    help="library's own stream-ordered pool instead of PyTorch's caching allocator")
     args = ap.parse_args()
     if args.warmup < 3:
         log("note: --warmup < 3 violates the timing rules; using 3")

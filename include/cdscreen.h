@@ -169,6 +169,17 @@ typedef struct {
                                  sets whose union is the unsharded result -- provided the
                                  elements passed are the shard's members (cd_shell_members: own
                                  objects plus the g_c halo above the band).  CD_GRID/CD_HYBRID. */
+    /* Device scratch memory of the call (PyTorch supplies memory).  When alloc and
+       free are set (both or neither: CD_EINVAL), every device buffer of the call -- orbit
+       records, grid arena, queues, sort scratch, results -- comes from alloc(bytes, alloc_ctx)
+       (NULL = out of memory -> CD_ENOMEM / CD_ECUDA) and is returned with free(p, alloc_ctx);
+       all use is ordered on the call's stream, so a stream-ordered caching allocator on that
+       stream (e.g. torch.cuda.caching_allocator_alloc) may reuse a freed block at once.  Device
+       results (outputs_on_device) are released with the same free in cd_conjunctions_free, so
+       the allocator must outlive them.  NULL (default): the device's stream-ordered pool.     */
+    void* (*alloc)(size_t bytes, void* ctx);
+    void (*free)(void* p, void* ctx);
+    void* alloc_ctx;
 } cd_options;
 
 /* Fill *opt with the defaults above. */

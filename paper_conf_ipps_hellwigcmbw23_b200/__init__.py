@@ -79,6 +79,10 @@ class cd_stats(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p)
+FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_void_p)
+
+
 class cd_options(C.Structure):
     _fields_ = [("v_margin", C.c_double), ("grid_origin", C.c_double * 3), ("device", C.c_int),
                 ("stream", C.c_void_p), ("rank", C.c_int), ("n_ranks", C.c_int),
@@ -87,7 +91,8 @@ class cd_options(C.Structure):
                 ("batch_object_steps", C.c_size_t), ("round_steps", C.c_size_t),
                 ("profile_phases", C.c_int), ("l2_persist", C.c_int), ("grid_table", C.c_int),
                 ("stats", C.POINTER(cd_stats)), ("propagator", C.c_int),
-                ("shell_lo", C.c_double), ("shell_hi", C.c_double)]
+                ("shell_lo", C.c_double), ("shell_hi", C.c_double),
+                ("alloc", ALLOC_FN), ("free", FREE_FN), ("alloc_ctx", C.c_void_p)]
 
 
 class cd_plan_info(C.Structure):
@@ -234,10 +239,46 @@ class _Elements:
         self.s = cd_elements(*ptrs)
 
 
+class TorchAllocator:
+    """cd_options.alloc / free backed by PyTorch's CUDA caching allocator on one device and
+    stream (the call's stream: all of the library's use of a block is ordered on it).  Keep the
+    object alive while the call runs and while device results from it exist."""
+
+    def __init__(self, device, stream):
+        import torch
+        self.device = int(device)
+        self.stream = stream
+        self.live = 0
+        self.peak = 0
+        self.calls = 0
+
+        def _alloc(nbytes, ctx):
+            try:
+                p = torch.cuda.caching_allocator_alloc(int(nbytes), self.device, self.stream)
+            except Exception:
+                return None
+            self.live += 1
+            self.calls += 1
+            self.peak = max(self.peak, self.live)
+            return p
+
+        def _free(p, ctx):
+            torch.cuda.caching_allocator_delete(p)
+            self.live -= 1
+
+        self.c_alloc = ALLOC_FN(_alloc)
+        self.c_free = FREE_FN(_free)
+
+    def install(self, opt):
+        opt.alloc = self.c_alloc
+        opt.free = self.c_free
+        opt.alloc_ctx = None
+
+
 def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None, stream=None,
                  cell_factor=None, batch_object_steps=None, round_steps=None,
                  outputs_on_device=False, inputs_on_device=False, profile_phases=False,
-                 l2_persist=None, grid_table=None, propagator=None, shell=None):
+                 l2_persist=None, grid_table=None, propagator=None, shell=None, allocator=None):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -267,6 +308,8 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
         o.propagator = PROPAGATORS[propagator] if isinstance(propagator, str) else int(propagator)
     if shell is not None:
         o.shell_lo, o.shell_hi = float(shell[0]), float(shell[1])
+    if allocator is not None:
+        allocator.install(o)
     return o
 
 
@@ -286,11 +329,24 @@ def _torch_stream():
     return None
 
 
+def _resolve_allocator(kw):
+    """allocator="torch": PyTorch's caching allocator on the current device and stream (the call
+    then runs on that stream)."""
+    if kw.get("allocator") == "torch":
+        import torch
+        dev = torch.cuda.current_device() if kw.get("device") is None else int(kw["device"])
+        stream = kw.get("stream") or torch.cuda.current_stream(dev).cuda_stream
+        kw["stream"] = stream
+        kw["allocator"] = TorchAllocator(dev, stream)
+    return kw.get("allocator")
+
+
 def screen(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
     """Conjunctions as a structured numpy array (CONJ_DTYPE), sorted by (i, j, step)."""
     E = _Elements(pop)
     st = cd_stats()
     kw.setdefault("propagator", E.propagator)
+    keep_alloc = _resolve_allocator(kw)   # noqa: F841 (alive for the call)
     opt = make_options(inputs_on_device=E.on_device, **kw)
     if opt.stream is None and E.on_device:
         opt.stream = _torch_stream()
@@ -315,6 +371,7 @@ def candidates(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
     E = _Elements(pop)
     st = cd_stats()
     kw.setdefault("propagator", E.propagator)
+    keep_alloc = _resolve_allocator(kw)   # noqa: F841
     opt = make_options(inputs_on_device=E.on_device, **kw)
     opt.stats = C.pointer(st)
     p = C.c_void_p()

@@ -74,7 +74,7 @@ cd_status fail(cd_status s, const char* fmt, ...)
         if (_s != CD_OK) return _s;     \
     } while (0)
 
-// stream-ordered device buffer
+// stream-ordered device buffer (dev_malloc: the caller's allocator or the stream-ordered pool)
 template <typename T>
 struct DBuf {
     T* p = nullptr;
@@ -87,7 +87,7 @@ struct DBuf {
     ~DBuf() { release(); }
     void release()
     {
-        if (p) cudaFreeAsync(p, st);
+        if (p) dev_free(p, st);
         p = nullptr;
         n = 0;
     }
@@ -95,7 +95,7 @@ struct DBuf {
     {
         release();
         n = count;
-        return cudaMallocAsync((void**)&p, sizeof(T) * (count ? count : 1), st);
+        return dev_malloc((void**)&p, sizeof(T) * (count ? count : 1), st);
     }
     T* detach()
     {
@@ -257,6 +257,7 @@ struct Owner {
     void* p;
     cudaStream_t st;   // device results: released stream-ordered on the call's stream
     size_t host_bytes; // host results: size of the anonymous mapping (munmap)
+    DevAlloc alloc;    // device results from the caller's allocator: released with its free
 };
 
 // Optional per-phase device timing (cd_options.profile_phases): CUDA events recorded on the
@@ -370,6 +371,7 @@ struct Call {
     PhaseTimer pt;
     ~Call()
     {
+        g_dev_alloc = DevAlloc{};
         if (ev0) cudaEventDestroy(ev0);
         if (ev1) cudaEventDestroy(ev1);
         if (own_stream && st) {
@@ -399,6 +401,7 @@ struct Call {
             return fail(CD_ENODEV, "libcdscreen is built for sm_100a (B200); device %d is sm_%d",
                         dev, cc);
         setup_pool(dev);
+        g_dev_alloc = DevAlloc{o.alloc, o.free, o.alloc_ctx};
         if (o.stream) {
             st = (cudaStream_t)o.stream;
         } else {
@@ -431,6 +434,8 @@ cd_status validate_scalars(size_t n, double t0, double t1, double dt, double d, 
         return fail(CD_EINVAL, "need 0 <= rank < n_ranks");
     if (o.propagator != CD_PROP_KEPLER && o.propagator != CD_PROP_J2)
         return fail(CD_EINVAL, "unknown propagator %d", o.propagator);
+    if ((o.alloc == nullptr) != (o.free == nullptr))
+        return fail(CD_EINVAL, "cd_options.alloc and free must be given together");
     if (!is_fin(o.shell_lo) || !is_fin(o.shell_hi) || o.shell_lo < 0.0 ||
         (o.shell_hi != 0.0 && !(o.shell_hi > o.shell_lo)))
         return fail(CD_EINVAL, "need shell_hi = 0 (no shard) or shell_hi > shell_lo >= 0");
@@ -596,19 +601,31 @@ struct ConjBuf {
     Conj* p = nullptr;
     size_t n = 0;
     std::vector<Conj*> retired;
+    DevAlloc user = g_dev_alloc;   // the caller's allocator, if the call has one
     ConjBuf() = default;
     ConjBuf(const ConjBuf&) = delete;
     ConjBuf& operator=(const ConjBuf&) = delete;
     ~ConjBuf()
     {
-        for (Conj* r : retired) cudaFree(r);
-        if (p) cudaFree(p);
+        for (Conj* r : retired) release(r);
+        if (p) release(p);
+    }
+    void release(Conj* q)
+    {
+        if (user.free) user.free(q, user.ctx);
+        else cudaFree(q);
     }
     // new buffer of `count` records; the first `keep` records are copied over (stream-ordered)
     cudaError_t grow(size_t count, size_t keep, cudaStream_t st)
     {
         Conj* np = nullptr;
-        cudaError_t e = cudaMalloc((void**)&np, sizeof(Conj) * (count ? count : 1));
+        cudaError_t e = cudaSuccess;
+        if (user.alloc) {
+            np = static_cast<Conj*>(user.alloc(sizeof(Conj) * (count ? count : 1), user.ctx));
+            if (!np) return cudaErrorMemoryAllocation;
+        } else {
+            e = cudaMalloc((void**)&np, sizeof(Conj) * (count ? count : 1));
+        }
         if (e != cudaSuccess) return e;
         if (p && keep) e = cudaMemcpyAsync(np, p, sizeof(Conj) * keep, cudaMemcpyDeviceToDevice, st);
         if (p) retired.push_back(p);
@@ -791,7 +808,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     if (want == Want::Conj) {
         Conj* cp = nullptr;
         size_t cc = 0;
-        if (conj_cache_take(C.dev, st, &cp, &cc) && cc >= ocap) {
+        if (!g_dev_alloc.alloc && conj_cache_take(C.dev, st, &cp, &cc) && cc >= ocap) {
             R.conj.p = cp;
             R.conj.n = cc;
             ocap = cc;
@@ -1198,10 +1215,12 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
         }
         // the accumulation buffer goes back to the per-device cache (its last use, the sort,
         // is enqueued on C.st)
+        // (with the caller's allocator it is simply released by R's destructor)
         const size_t cap = R.conj.n;
-        conj_cache_give(C.dev, C.st, R.conj.detach(), cap);
+        if (!R.conj.user.alloc) conj_cache_give(C.dev, C.st, R.conj.detach(), cap);
     }
-    Owner* own = new Owner{o.outputs_on_device != 0, nullptr, C.own_stream ? nullptr : C.st, 0};
+    Owner* own = new Owner{o.outputs_on_device != 0, nullptr, C.own_stream ? nullptr : C.st, 0,
+                           g_dev_alloc};
     if (R.n_conj) {
         if (o.outputs_on_device) {
             own->p = sorted.detach();
@@ -1409,7 +1428,8 @@ void cd_conjunctions_free(cd_conjunctions* c)
             // stream-ordered release (no device-wide synchronisation): after the work the
             // caller queued on the call's stream (the legacy default stream if the library
             // created its own)
-            if (own->device) cudaFreeAsync(own->p, own->st);
+            if (own->device && own->alloc.free) own->alloc.free(own->p, own->alloc.ctx);
+            else if (own->device) cudaFreeAsync(own->p, own->st);
             else munmap(own->p, own->host_bytes);
         }
         delete own;

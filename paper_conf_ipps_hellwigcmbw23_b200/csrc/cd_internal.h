@@ -18,6 +18,33 @@ struct LaunchCount {
     void bump(uint64_t k = 1) { n += k; g_launches.fetch_add(k, std::memory_order_relaxed); }
 };
 
+// Device scratch memory of the current call (thread-local, set by the call for its duration):
+// the caller's allocator (cd_options.alloc / free / alloc_ctx, e.g. PyTorch's caching allocator)
+// when given, else the device's stream-ordered pool.
+struct DevAlloc {
+    void* (*alloc)(size_t bytes, void* ctx) = nullptr;
+    void (*free)(void* p, void* ctx) = nullptr;
+    void* ctx = nullptr;
+};
+extern thread_local DevAlloc g_dev_alloc;
+
+inline cudaError_t dev_malloc(void** p, size_t bytes, cudaStream_t st)
+{
+    if (bytes == 0) bytes = 1;
+    if (g_dev_alloc.alloc) {
+        *p = g_dev_alloc.alloc(bytes, g_dev_alloc.ctx);
+        return *p ? cudaSuccess : cudaErrorMemoryAllocation;
+    }
+    return cudaMallocAsync(p, bytes, st);
+}
+
+inline void dev_free(void* p, cudaStream_t st)
+{
+    if (!p) return;
+    if (g_dev_alloc.free) g_dev_alloc.free(p, g_dev_alloc.ctx);
+    else cudaFreeAsync(p, st);
+}
+
 struct Elements {   // device pointers (external order)
     const double *a, *e, *inc, *raan, *argp, *nu0;
 };

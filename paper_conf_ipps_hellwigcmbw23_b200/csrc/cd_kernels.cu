@@ -16,6 +16,7 @@ using namespace cdk;
 namespace cdh {
 
 std::atomic<uint64_t> g_launches{0};
+thread_local DevAlloc g_dev_alloc;
 
 static inline unsigned blocks_for(int64_t n, int t) { return (unsigned)((n + t - 1) / t); }
 

@@ -18,7 +18,7 @@ namespace cdh {
 template <typename T>
 static cudaError_t dalloc(T** p, size_t count, cudaStream_t st)
 {
-    return cudaMallocAsync((void**)p, sizeof(T) * (count ? count : 1), st);
+    return dev_malloc((void**)p, sizeof(T) * (count ? count : 1), st);
 }
 
 cudaError_t sort_pairs_u32(const uint32_t* kin, uint32_t* kout, const uint32_t* vin, uint32_t* vout,
@@ -28,11 +28,12 @@ cudaError_t sort_pairs_u32(const uint32_t* kin, uint32_t* kout, const uint32_t* 
     CD_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, kin, kout, vin, vout, (int64_t)count,
                                            0, end_bit, st));
     void* tmp = nullptr;
-    CD_TRY(cudaMallocAsync(&tmp, tmp_bytes ? tmp_bytes : 1, st));
+    CD_TRY(dev_malloc(&tmp, tmp_bytes ? tmp_bytes : 1, st));
     CD_TRY(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, kin, kout, vin, vout, (int64_t)count, 0,
                                            end_bit, st));
     lc.bump(4);   // CUB onesweep: histogram + exclusive scan + one pass per 8-bit digit (upper bound)
-    return cudaFreeAsync(tmp, st);
+    dev_free(tmp, st);
+    return cudaGetLastError();
 }
 
 template <typename Rec>
@@ -97,7 +98,7 @@ static cudaError_t finalize_impl(const Rec* in, size_t n, const uint32_t* perm, 
     CD_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb2, k2, k2o, i1o, i2o, (int64_t)n, 0, 64, st));
     if (tb2 > tb) tb = tb2;
     void* tmp = nullptr;
-    CD_TRY(cudaMallocAsync(&tmp, tb ? tb : 1, st));
+    CD_TRY(dev_malloc(&tmp, tb ? tb : 1, st));
     CD_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, k1, k1o, i1, i1o, (int64_t)n, 0, 32, st));
     lc.bump(6);
     // pass 2 (stable): by (i, j) in caller ids
@@ -109,14 +110,14 @@ static cudaError_t finalize_impl(const Rec* in, size_t n, const uint32_t* perm, 
     k_gather<Rec><<<blocks, 256, 0, st>>>(in, i2o, n, perm, out);
     lc.bump();
     CD_TRY(cudaGetLastError());
-    cudaFreeAsync(tmp, st);
-    cudaFreeAsync(k1, st);
-    cudaFreeAsync(k1o, st);
-    cudaFreeAsync(i1, st);
-    cudaFreeAsync(i1o, st);
-    cudaFreeAsync(i2o, st);
-    cudaFreeAsync(k2, st);
-    cudaFreeAsync(k2o, st);
+    dev_free(tmp, st);
+    dev_free(k1, st);
+    dev_free(k1o, st);
+    dev_free(i1, st);
+    dev_free(i1o, st);
+    dev_free(i2o, st);
+    dev_free(k2, st);
+    dev_free(k2o, st);
     return cudaGetLastError();
 }
 
