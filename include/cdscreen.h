@@ -117,11 +117,15 @@ typedef struct {
 typedef struct {
     uint64_t steps;            /* sampling steps screened by this call (this rank's slice)    */
     uint64_t object_steps;     /* n * steps                                                    */
-    uint64_t candidates;       /* |K| for this slice (hybrid: coarse candidates)              */
+    uint64_t candidates;       /* |K| for this slice (hybrid: coarse candidates; legacy: pairs
+                                  screened by this rank)                                      */
     uint64_t refined;          /* candidates that survived the conservative linear pre-filter
-                                  (hybrid: time-window work items + coplanar candidates)     */
+                                  (hybrid: time-window work items + coplanar candidates;
+                                  legacy: surviving time-window intervals)                    */
     uint64_t conjunctions;     /* reported rows                                               */
     uint64_t hybrid_ap_rejected, hybrid_coplanar, hybrid_path_rejected, hybrid_time_rejected;
+                               /* filter-stage counts (hybrid: per coarse candidate; legacy:
+                                  per pair)                                                   */
     uint64_t kernel_launches;  /* CUDA kernels launched by this call                          */
     uint64_t retries;          /* capacity-overflow retries                                   */
     double ms_total;           /* device time of the call (CUDA events on the call's stream)  */

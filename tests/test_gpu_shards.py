@@ -74,3 +74,16 @@ def test_shard_option_errors():
     with pytest.raises(cds.CdError) as ei:
         cds.screen(pop, 0.0, 10.0, 1.0, 2.0, mode="legacy", shell=(0.0, 7000.0))
     assert ei.value.status == cds.CD_EINVAL
+
+
+def test_shards_times_slices():
+    """The two sharding axes combine (rank = (shard, time slice)): 3 radial shards x 4 time
+    slices partition the result exactly."""
+    pop = popgen.random_population(20000, 78, "catalog", 4000)
+    t0, t1, dt, d = 500.0, 899.0, 1.0, 5.0
+    whole = cds.screen(pop, t0, t1, dt, d)
+    b = cdist.shell_bounds(pop, 3)
+    parts = [cdist.screen_shard(pop, t0, t1, dt, d, b, s, rank=q, n_ranks=4)[0]
+             for s in range(3) for q in range(4)]
+    assert len(whole) > 50
+    assert np.array_equal(_union(parts), whole)
