@@ -556,14 +556,18 @@ enum class Want { Conj, Cand };
 // the objects of those cells (~ (m + 2)^3 x density, or 27 x density / 2 in half-shell mode);
 // a walked object costs about 1.5 probes.  Only performance depends on m (any L >= g_c gives
 // the same candidate set).
+#ifndef CD_WALK_WEIGHT
+#define CD_WALK_WEIGHT 3.0
+#endif
 double choose_cell_factor(double c)
 {
     const double dens = 2.0 * c / 4.18879;
-    double best = 1.0, bestcost = 13.0 + 1.5 * 13.5 * dens;
+    const double w = CD_WALK_WEIGHT;   // cost of one walked list entry relative to one probe
+    double best = 1.0, bestcost = 13.0 + w * 13.5 * dens;
     const double cand[] = {2.0, 3.0, 4.0, 5.0, 6.0, 8.0};
     for (double m : cand) {
         const double probes = std::pow(1.0 + 2.0 / m, 3.0) - 1.0;
-        const double cost = probes + 1.5 * std::pow(m + 2.0, 3.0) * dens;
+        const double cost = probes + w * std::pow(m + 2.0, 3.0) * dens;
         if (cost < bestcost) {
             bestcost = cost;
             best = m;
@@ -737,7 +741,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     // can follow the cell edge chosen after the first round.
     const bool can_chain = o.grid_table != 1, can_open = o.grid_table != 2;
 #ifndef CD_CHAIN_FACTOR
-#define CD_CHAIN_FACTOR 4
+#define CD_CHAIN_FACTOR 8
 #endif
     const uint64_t chain_words = can_chain ? std::max<uint64_t>(next_pow2((uint64_t)n * CD_CHAIN_FACTOR), 1024) : 0;
     const uint64_t nbits = std::max<uint64_t>(next_pow2((uint64_t)n * 32), 1024);   // open: >= 32 bits/object
@@ -1476,7 +1480,7 @@ cd_status cd_plan(size_t n, double t0, double t1, double dt, double d, cd_mode m
         // 32-byte entries {x, y, z, next}
         const double m = choose_cell_factor(std::max(1.0, out->est_candidates_per_step) / std::max(1.0, nn));
         const double n_u = std::max(1.0, nn);
-        const double chained = 4.0 * (double)next_pow2((uint64_t)(4.0 * n_u));
+        const double chained = 4.0 * (double)next_pow2((uint64_t)(CD_CHAIN_FACTOR * n_u));
         const double open = 16.0 * (double)next_pow2((uint64_t)(2.0 * n_u)) +
                             (double)next_pow2((uint64_t)(32.0 * n_u)) / 8.0;
         out->bytes_per_grid = (m < 2.0 ? open : chained) + 32.0 * nn;
