@@ -82,14 +82,20 @@ __global__ void __launch_bounds__(256, CD_FILTER_MINB) k_hybrid_filter(Orbits O,
             const double sg = node ? -1.0 : 1.0;   // mutual node / opposite node (f + pi)
             if (node_closed(A, B, d, gA, gB, sg)) continue;   // orbit path: node closed
             any_node = true;
-            double atl, ath, btl, bth;
-            node_window(A, gA, sg, atl, ath);
-            node_window(B, gB, sg, btl, bth);
             // the copies k T of each periodic window that meet the owner cell [lo, hi] (windows
             // are shorter than half a period and the cell far shorter than a period: at most two
-            // of three consecutive copies), intersected pairwise
+            // of three consecutive copies), intersected pairwise.  A's window first: B's is only
+            // computed when one of A's copies meets the cell (most pairs end here)
+            double atl, ath, btl, bth;
+            node_window(A, gA, sg, atl, ath);
             const double TA = kTwoPiH / A.nm, TB = kTwoPiH / B.nm;
-            const double ka = floor((lo - (ath - tk)) / TA), kb = floor((lo - (bth - tk)) / TB);
+            const double ka = floor((lo - (ath - tk)) / TA);
+            bool a_meets = false;
+            for (int x = 0; x < 3; ++x)
+                a_meets = a_meets || fmin(ath - tk + (ka + x) * TA, hi) >= fmax(atl - tk + (ka + x) * TA, lo);
+            if (!a_meets) continue;
+            node_window(B, gB, sg, btl, bth);
+            const double kb = floor((lo - (bth - tk)) / TB);
             for (int x = 0; x < 3; ++x) {
                 const double al = fmax(atl - tk + (ka + x) * TA, lo), ah = fmin(ath - tk + (ka + x) * TA, hi);
                 if (!(ah >= al)) continue;
