@@ -289,18 +289,19 @@ __constant__ int8_t kHalfShell[14][3] = {
     {0, 1, -1}, {0, 1, 0}, {0, 1, 1},
     {0, 0, 1}};
 
-// Block-level candidate staging (role-C blocks of k_step, GridGeom::stage): candidates are
-// appended to a shared buffer with a shared-memory atomic and flushed to the global queue with
-// one global atomic per block; a full buffer falls back to the warp-aggregated global append.
-// A dense coarse grid (the hybrid's 1.4 candidates per object-step) otherwise serialises on the
-// queue counter (hybrid k_step 556 -> 284 us per 1M-object step); a sparse one (the grid
-// variant's 0.004) does not need it and skips the block barriers (64 vs 68 us).
+// Warp-level candidate staging (role-C warps of k_step, GridGeom::stage): each warp appends its
+// candidates to its own slice of a shared buffer with a shared-memory atomic and flushes them to
+// the global queue with one global atomic per warp; a full slice falls back to the
+// warp-aggregated global append.  A dense coarse grid (the hybrid's 1.4 candidates per
+// object-step) otherwise serialises on the queue counter (hybrid k_step 556 -> 284 us per
+// 1M-object step with block-level staging, and a warp-level flush drops the block barrier at the
+// end); a sparse one (the grid variant's 0.004) does not need it.
 // The buffer is dynamic shared memory, requested only for staged launches: a sparse step keeps
 // the whole L1 (static shared memory here cost the grid variant 3 %).
-constexpr unsigned kSCand = 1024;
+constexpr unsigned kSCand = 1024;              // per block (256 threads)
+constexpr unsigned kSWarp = kSCand / 8;        // per warp
 extern __shared__ Cand s_cand[];
-__shared__ unsigned s_ncand;
-__shared__ unsigned long long s_cbase;
+__shared__ unsigned s_nw[8];
 
 __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_t j, const double p[3],
                                           const Entry& ej, uint32_t step, Cand* __restrict__ q,
@@ -319,9 +320,10 @@ __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_
         cd.j = r < j ? j : r;
         cd.step = step;
         if (g.stage) {
-            const unsigned k = atomicAdd(&s_ncand, 1u);
-            if (k < kSCand) {
-                s_cand[k] = cd;
+            const unsigned w = threadIdx.x >> 5;
+            const unsigned k = atomicAdd(&s_nw[w], 1u);
+            if (k < kSWarp) {
+                s_cand[w * kSWarp + k] = cd;
                 return;
             }
         }
@@ -606,9 +608,10 @@ __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
         const int s = (int)(b3 / nbC);
         const int64_t r = (int64_t)(b3 % nbC) * 256 + threadIdx.x;
         const bool stage = a.g.stage != 0;   // uniform over the launch
+        const unsigned lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
         if (stage) {
-            if (threadIdx.x == 0) s_ncand = 0;
-            __syncthreads();
+            if (lane == 0) s_nw[wid] = 0;
+            __syncwarp();
         }
         if (r < a.O.n) {
             if (kChained)
@@ -619,15 +622,16 @@ __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
                         a.qcap, a.ctrl);
         }
         if (!stage) return;
-        // flush the block's staged candidates: one global atomic, coalesced copy
-        __syncthreads();
-        const unsigned m = min(s_ncand, kSCand);
+        // flush the warp's staged candidates: one global atomic, coalesced copy
+        __syncwarp();
+        const unsigned m = min(s_nw[wid], kSWarp);
         if (m == 0) return;
-        if (threadIdx.x == 0) s_cbase = atomicAdd(&a.ctrl->n_cand, (unsigned long long)m);
-        __syncthreads();
-        for (unsigned k = threadIdx.x; k < m; k += 256) {
-            const unsigned long long idx = s_cbase + k;
-            if (idx < a.qcap) a.q[idx] = s_cand[k];
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(&a.ctrl->n_cand, (unsigned long long)m);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        for (unsigned k = lane; k < m; k += 32) {
+            const unsigned long long idx = base + k;
+            if (idx < a.qcap) a.q[idx] = s_cand[wid * kSWarp + k];
         }
     }
 }
