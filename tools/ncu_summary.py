@@ -14,7 +14,10 @@ WANT = ['gpu__time_duration.sum', 'dram__bytes_read.sum', 'dram__bytes_write.sum
         'l1tex__t_sector_hit_rate.pct', 'sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active',
         'smsp__inst_executed.sum', 'smsp__average_warp_latency_per_inst_issued.ratio',
         'smsp__warps_eligible.avg.per_cycle_active', 'smsp__issue_active.avg.pct_of_peak_sustained_active',
-        'lts__t_sectors_op_atom.sum', 'lts__t_sectors_op_red.sum', 'l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum',
+        'lts__t_sectors_op_atom.sum', 'lts__t_sectors_op_red.sum',
+        'l1tex__m_l1tex2xbar_write_sectors_mem_global_op_atom.sum',
+        'l1tex__m_l1tex2xbar_write_sectors_mem_global_op_atom.sum.per_second',
+        'l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum',
         'l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum',
         'smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio',
         'smsp__average_warps_issue_stalled_lg_throttle_per_issue_active.ratio',
