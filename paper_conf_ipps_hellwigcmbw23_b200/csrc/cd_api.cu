@@ -557,7 +557,7 @@ enum class Want { Conj, Cand };
 // a walked object costs about 1.5 probes.  Only performance depends on m (any L >= g_c gives
 // the same candidate set).
 #ifndef CD_WALK_WEIGHT
-#define CD_WALK_WEIGHT 3.0
+#define CD_WALK_WEIGHT 5.0
 #endif
 double choose_cell_factor(double c)
 {
