@@ -92,7 +92,8 @@ class cd_options(C.Structure):
                 ("profile_phases", C.c_int), ("l2_persist", C.c_int), ("grid_table", C.c_int),
                 ("stats", C.POINTER(cd_stats)), ("propagator", C.c_int),
                 ("shell_lo", C.c_double), ("shell_hi", C.c_double),
-                ("alloc", ALLOC_FN), ("free", FREE_FN), ("alloc_ctx", C.c_void_p)]
+                ("alloc", ALLOC_FN), ("free", FREE_FN), ("alloc_ctx", C.c_void_p),
+                ("shards", C.c_int)]
 
 
 class cd_plan_info(C.Structure):
@@ -278,7 +279,8 @@ class TorchAllocator:
 def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None, stream=None,
                  cell_factor=None, batch_object_steps=None, round_steps=None,
                  outputs_on_device=False, inputs_on_device=False, profile_phases=False,
-                 l2_persist=None, grid_table=None, propagator=None, shell=None, allocator=None):
+                 l2_persist=None, grid_table=None, propagator=None, shell=None, allocator=None,
+                 shards=None):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -310,6 +312,8 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
         o.shell_lo, o.shell_hi = float(shell[0]), float(shell[1])
     if allocator is not None:
         allocator.install(o)
+    if shards is not None:
+        o.shards = int(shards)
     return o
 
 

@@ -434,6 +434,7 @@ cd_status validate_scalars(size_t n, double t0, double t1, double dt, double d, 
         return fail(CD_EINVAL, "need 0 <= rank < n_ranks");
     if (o.propagator != CD_PROP_KEPLER && o.propagator != CD_PROP_J2)
         return fail(CD_EINVAL, "unknown propagator %d", o.propagator);
+    if (o.shards < 0 || o.shards > 64) return fail(CD_EINVAL, "need 0 <= shards <= 64");
     if ((o.alloc == nullptr) != (o.free == nullptr))
         return fail(CD_EINVAL, "cd_options.alloc and free must be given together");
     if (!is_fin(o.shell_lo) || !is_fin(o.shell_hi) || o.shell_lo < 0.0 ||
@@ -1071,7 +1072,13 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             if (L < gc * (1.0 + 1e-12)) L = gc * (1.0 + 1e-12);
             g.inv_cell = 1.0 / L;
             g.halfshell = L < 2.0 * gc ? 1 : 0;
+            const bool was_chained = chained;
             chained = pick_chained(g);
+            if (chained != was_chained) {
+                // the bitmap / head sets change meaning (occupancy bits <-> epoch-tagged list
+                // heads): clear all three, stream-ordered after the round already in flight
+                CU(cudaMemsetAsync(bitset[0], 0, 3 * bit_bytes, st));
+            }
             settled = true;
         }
         if (!o.round_steps) {
@@ -1170,6 +1177,123 @@ cd_status run_legacy(Call& C, const OrbitSet& S, double t0, double t1, double dt
     return CD_OK;
 }
 
+// Radial L2 shards (cd_options.shards; SURVEY 8(f) row 2 applied on one device): a large
+// population's per-step grid (~64 B per object) overflows the 126 MB L2 and the scan turns into
+// DRAM-latency-bound random access.  The objects are split into S radial bands (quantiles of a);
+// each band is screened in turn with only its members (cd_shell_members' rule: own band + g_c
+// halo above it) and keeps the candidates whose smaller radius lies in the band, so the union of
+// the bands' results is exactly the unsharded result (tests/test_gpu_shards.py).  Measured at
+// 8M objects: 300 steps 1.09 -> 0.84 s with 2 bands (tools/shard_probe.py); no gain at 1M.
+int shard_count(const cd_options& o, size_t n, cd_mode mode)
+{
+    if (mode == CD_LEGACY || o.shell_hi != 0.0) return 1;
+    if (o.shards > 0) return o.shards;
+    if (n < 3000000) return 1;
+    return (int)std::max<size_t>(2, (n + 2000000) / 4000000);
+}
+
+cd_status screen_sharded(Call& C, const cd_elements* el, size_t n, double t0, double t1, double dt,
+                         double d, cd_mode mode, const cd_options& o, int64_t K, int S,
+                         DBuf<Conj>& sorted, size_t& nconj, cd_stats& stats)
+{
+    cudaStream_t st = C.st;
+    if (!el || !el->a || !el->e || !el->inc || !el->raan || !el->argp || !el->nu0)
+        return fail(CD_EINVAL, "elements must be non-NULL");
+    // the full element set on the device once (validated), a and e on the host for the bands
+    DBuf<double> up(st);
+    Elements E;
+    std::vector<double> ha(n), he(n);
+    if (o.inputs_on_device) {
+        E = Elements{el->a, el->e, el->inc, el->raan, el->argp, el->nu0};
+        CU(cudaMemcpyAsync(ha.data(), el->a, sizeof(double) * n, cudaMemcpyDeviceToHost, st));
+        CU(cudaMemcpyAsync(he.data(), el->e, sizeof(double) * n, cudaMemcpyDeviceToHost, st));
+        CU(cudaStreamSynchronize(st));
+    } else {
+        const double* src[6] = {el->a, el->e, el->inc, el->raan, el->argp, el->nu0};
+        TRY(validate_elements_host(src, n));
+        CU(up.alloc(6 * n));
+        for (int c = 0; c < 6; ++c)
+            CU(cudaMemcpyAsync(up.p + c * n, src[c], sizeof(double) * n, cudaMemcpyHostToDevice, st));
+        E = Elements{up.p, up.p + n, up.p + 2 * n, up.p + 3 * n, up.p + 4 * n, up.p + 5 * n};
+        memcpy(ha.data(), el->a, sizeof(double) * n);
+        memcpy(he.data(), el->e, sizeof(double) * n);
+    }
+    // band edges: quantiles of a (strictly increasing; duplicates merge bands)
+    std::vector<double> edges{0.0};
+    {
+        std::vector<double> tmp = ha;
+        for (int s = 1; s < S; ++s) {
+            const size_t k = n * (size_t)s / (size_t)S;
+            std::nth_element(tmp.begin(), tmp.begin() + k, tmp.end());
+            if (tmp[k] > edges.back()) edges.push_back(tmp[k]);
+        }
+        edges.push_back(1.0e9);
+    }
+    const double gc = d + o.v_margin * dt;
+    DBuf<Conj> all(st);
+    size_t nall = 0;
+    std::vector<uint32_t> idx;
+    idx.reserve(n);
+    for (size_t s = 0; s + 1 < edges.size(); ++s) {
+        const double lo = edges[s], hi = edges[s + 1];
+        idx.clear();
+        for (size_t i = 0; i < n; ++i)
+            if (ha[i] * (1.0 + he[i]) >= lo && ha[i] * (1.0 - he[i]) < hi + gc) idx.push_back((uint32_t)i);
+        const int64_t m = (int64_t)idx.size();
+        if (m < 2) continue;
+        DBuf<uint32_t> didx(st);
+        CU(didx.alloc((size_t)m));
+        CU(cudaMemcpyAsync(didx.p, idx.data(), sizeof(uint32_t) * (size_t)m, cudaMemcpyHostToDevice, st));
+        DBuf<double> sub(st);
+        CU(sub.alloc(6 * (size_t)m));
+        CU(launch_gather_elements(E, didx.p, m, sub.p, st, C.lc));
+        const cd_elements sel{sub.p, sub.p + m, sub.p + 2 * m, sub.p + 3 * m, sub.p + 4 * m, sub.p + 5 * m};
+        cd_options os = o;
+        os.inputs_on_device = 1;
+        os.shell_lo = lo;
+        os.shell_hi = hi;
+        OrbitSet Ss;
+        TRY(prepare_orbits(C, &sel, (size_t)m, os, Ss));
+        CU(launch_compose_perm(Ss.perm.p, didx.p, m, st, C.lc));   // internal -> global ids
+        Result Rs;
+        cd_stats ss;
+        memset(&ss, 0, sizeof ss);
+        TRY(run(C, Ss, t0, t1, dt, d, mode, os, K, Want::Conj, Rs, ss));
+        stats.candidates += ss.candidates;
+        stats.refined += ss.refined;
+        stats.retries += ss.retries;
+        stats.hybrid_ap_rejected += ss.hybrid_ap_rejected;
+        stats.hybrid_coplanar += ss.hybrid_coplanar;
+        stats.hybrid_path_rejected += ss.hybrid_path_rejected;
+        stats.hybrid_time_rejected += ss.hybrid_time_rejected;
+        stats.steps = ss.steps;
+        if (Rs.n_conj) {
+            if (nall + Rs.n_conj > all.n) {
+                DBuf<Conj> grown(st);
+                CU(grown.alloc(std::max(2 * all.n, nall + Rs.n_conj)));
+                if (nall) CU(cudaMemcpyAsync(grown.p, all.p, sizeof(Conj) * nall, cudaMemcpyDeviceToDevice, st));
+                const size_t cap = grown.n;
+                all.release();
+                all.p = grown.detach();
+                all.n = cap;
+            }
+            CU(launch_conj_to_global(Rs.conj.p, Rs.n_conj, Ss.perm.p, all.p + nall, st, C.lc));
+            nall += Rs.n_conj;
+        }
+        const size_t cap = Rs.conj.n;
+        if (!Rs.conj.user.alloc) conj_cache_give(C.dev, st, Rs.conj.detach(), cap);
+    }
+    stats.object_steps = stats.steps * (uint64_t)n;
+    nconj = nall;
+    if (nall) {
+        C.pt.start(kPhFinalize);
+        CU(sorted.alloc(nall));
+        CU(finalize_conj(all.p, nall, nullptr, sorted.p, st, C.lc));
+        C.pt.stop();
+    }
+    return CD_OK;
+}
+
 cd_options defaults()
 {
     cd_options o;
@@ -1203,7 +1327,12 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
     DBG("screen: begin");
     Result R;
     DBuf<Conj> sorted(C.st);
-    {
+    const int n_shards = n > 1 ? shard_count(o, n, mode) : 1;
+    if (n_shards > 1) {
+        size_t nc = 0;
+        TRY(screen_sharded(C, el, n, t0, t1, dt, d, mode, o, K, n_shards, sorted, nc, stats));
+        R.n_conj = nc;
+    } else {
         OrbitSet S;
         if (n > 0) TRY(prepare_orbits(C, el, n, o, S));
         else if (!el) return fail(CD_EINVAL, "elements must be non-NULL");

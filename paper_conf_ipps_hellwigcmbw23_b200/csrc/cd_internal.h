@@ -76,6 +76,14 @@ cudaError_t launch_propagate_out(const cdk::Orbits& O, const uint32_t* perm, con
                                  int64_t nt, double* xyz, double* vxyz, cudaStream_t st,
                                  LaunchCount& lc);
 
+// ---- radial L2 shards (screen_sharded) ----------------------------------------------------
+cudaError_t launch_gather_elements(const Elements& src, const uint32_t* idx, int64_t m, double* dst,
+                                   cudaStream_t st, LaunchCount& lc);
+cudaError_t launch_compose_perm(uint32_t* perm, const uint32_t* idx, int64_t m, cudaStream_t st,
+                                LaunchCount& lc);
+cudaError_t launch_conj_to_global(const cdk::Conj* in, size_t n, const uint32_t* perm,
+                                  cdk::Conj* out, cudaStream_t st, LaunchCount& lc);
+
 // ---- grid build + scan (a2-a6) ---------------------------------------------------------
 cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long long v,
                             cudaStream_t st, LaunchCount& lc);

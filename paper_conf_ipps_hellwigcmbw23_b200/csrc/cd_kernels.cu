@@ -181,6 +181,68 @@ cudaError_t launch_propagate_out(const Orbits& O, const uint32_t* perm, const do
 }
 
 // ---------------------------------------------------------------------------------------
+// radial L2 shards (screen_sharded in cd_api.cu): member gather, id composition, id mapping
+// ---------------------------------------------------------------------------------------
+__global__ void k_gather_elements(Elements src, const uint32_t* __restrict__ idx, int64_t m,
+                                  double* __restrict__ dst)
+{
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (r >= m) return;
+    const uint32_t i = idx[r];
+    dst[r] = src.a[i];
+    dst[m + r] = src.e[i];
+    dst[2 * m + r] = src.inc[i];
+    dst[3 * m + r] = src.raan[i];
+    dst[4 * m + r] = src.argp[i];
+    dst[5 * m + r] = src.nu0[i];
+}
+
+__global__ void k_compose_perm(uint32_t* __restrict__ perm, const uint32_t* __restrict__ idx, int64_t m)
+{
+    const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (r < m) perm[r] = idx[perm[r]];
+}
+
+__global__ void k_conj_to_global(const Conj* __restrict__ in, size_t n, const uint32_t* __restrict__ perm,
+                                 Conj* __restrict__ out)
+{
+    const size_t k = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
+    if (k >= n) return;
+    Conj c = in[k];
+    const uint32_t a = perm[c.i], b = perm[c.j];
+    c.i = a < b ? a : b;
+    c.j = a < b ? b : a;
+    out[k] = c;
+}
+
+cudaError_t launch_gather_elements(const Elements& src, const uint32_t* idx, int64_t m, double* dst,
+                                   cudaStream_t st, LaunchCount& lc)
+{
+    if (m <= 0) return cudaSuccess;
+    k_gather_elements<<<blocks_for(m, 256), 256, 0, st>>>(src, idx, m, dst);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_compose_perm(uint32_t* perm, const uint32_t* idx, int64_t m, cudaStream_t st,
+                                LaunchCount& lc)
+{
+    if (m <= 0) return cudaSuccess;
+    k_compose_perm<<<blocks_for(m, 256), 256, 0, st>>>(perm, idx, m);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_conj_to_global(const Conj* in, size_t n, const uint32_t* perm, Conj* out,
+                                  cudaStream_t st, LaunchCount& lc)
+{
+    if (n == 0) return cudaSuccess;
+    k_conj_to_global<<<blocks_for((int64_t)n, 256), 256, 0, st>>>(in, n, perm, out);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------------------
 // a4 helper: clear hash tables to the empty marker ("initialized with this value")
 // ---------------------------------------------------------------------------------------
 __global__ void k_fill_u64(ulonglong2* __restrict__ p, size_t n2, unsigned long long v)

@@ -87,3 +87,23 @@ def test_shards_times_slices():
              for s in range(3) for q in range(4)]
     assert len(whole) > 50
     assert np.array_equal(_union(parts), whole)
+
+
+@pytest.mark.parametrize("mode,dt,prop,S", [("grid", 1.0, "kepler", 2), ("grid", 1.0, "kepler", 5),
+                                            ("hybrid", 9.0, "kepler", 3), ("grid", 1.0, "j2", 3)])
+def test_library_l2_shards_equal_unsharded(mode, dt, prop, S):
+    """cd_options.shards: the library screens S radial bands in turn on one device; the result is
+    identical, field by field, to the unsharded call (and the default auto mode is off here)."""
+    import torch
+    pop = dict(popgen.random_population(30000, 79, "catalog", 6000), propagator=prop)
+    t0, t1, d = 2000.0, 2000.0 + 250 * dt, 5.0
+    one = cds.screen(pop, t0, t1, dt, d, mode=mode, shards=1)
+    auto = cds.screen(pop, t0, t1, dt, d, mode=mode)
+    many, st = cds.screen(pop, t0, t1, dt, d, mode=mode, shards=S, return_stats=True)
+    assert len(one) > 50
+    assert np.array_equal(auto, one)
+    assert np.array_equal(many, one)
+    tp = {k: torch.from_numpy(v).cuda() for k, v in pop.items() if k != "propagator"}
+    tp["propagator"] = prop
+    dev = cds.screen(tp, t0, t1, dt, d, mode=mode, shards=S, allocator="torch")
+    assert np.array_equal(dev, one)
