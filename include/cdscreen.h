@@ -184,13 +184,13 @@ typedef struct {
     void* (*alloc)(size_t bytes, void* ctx);
     void (*free)(void* p, void* ctx);
     void* alloc_ctx;
-    int shards;               /* radial L2 shards screened in turn on this device (CD_GRID and
-                                 CD_HYBRID without a shell band): a large population's per-step
-                                 grid (~64 B per object) overflows L2, so its objects are split
-                                 into radial bands (quantiles of a), each screened with only its
-                                 members (the shell_lo/hi rule) -- the union is exactly the
-                                 unsharded result.  0 = auto (1 below 3M objects, else
-                                 max(2, round(n / 4M))), 1 = off, <= 64                         */
+    int shards;               /* radial shards screened in turn on this device (CD_GRID and
+                                 CD_HYBRID without a shell band): the objects are split into S
+                                 radial bands (quantiles of a), each screened with only its
+                                 members (the shell_lo/hi rule), so a call's grid memory scales
+                                 with n/S plus the halo; the union is exactly the unsharded
+                                 result.  0 or 1 = off (default; at 8M objects on one B200 the
+                                 bands were measured 1-14 % slower), <= 64                        */
 } cd_options;
 
 /* Fill *opt with the defaults above. */

@@ -1177,19 +1177,22 @@ cd_status run_legacy(Call& C, const OrbitSet& S, double t0, double t1, double dt
     return CD_OK;
 }
 
-// Radial L2 shards (cd_options.shards; SURVEY 8(f) row 2 applied on one device): a large
-// population's per-step grid (~64 B per object) overflows the 126 MB L2 and the scan turns into
-// DRAM-latency-bound random access.  The objects are split into S radial bands (quantiles of a);
+// Radial shards screened in turn on one device (cd_options.shards; SURVEY 8(f) row 2 applied
+// on one device): a large population's per-step grid (~64 B per object) overflows the 126 MB L2
+// and the scan turns into DRAM-latency-bound random access, and a population beyond HBM needs
+// its grid split.  The objects are split into S radial bands (quantiles of a);
 // each band is screened in turn with only its members (cd_shell_members' rule: own band + g_c
 // halo above it) and keeps the candidates whose smaller radius lies in the band, so the union of
-// the bands' results is exactly the unsharded result (tests/test_gpu_shards.py).  Measured at
-// 8M objects: 300 steps 1.09 -> 0.84 s with 2 bands (tools/shard_probe.py); no gain at 1M.
+// the bands' results is exactly the unsharded result (tests/test_gpu_shards.py).  Measured on
+// one B200 at 8M objects (tools/shard_sweep.py, device-resident inputs, tuned cell edge): 1407
+// us per step unsharded, 1456 / 1427 / 1608 with 2 / 3 / 4 bands -- the halo and the eccentric
+// objects replicated into every band cost what the smaller grid saves -- so the default is off;
+// the option bounds the per-call grid memory (a band holds ~n/S objects plus its halo).
 int shard_count(const cd_options& o, size_t n, cd_mode mode)
 {
+    (void)n;
     if (mode == CD_LEGACY || o.shell_hi != 0.0) return 1;
-    if (o.shards > 0) return o.shards;
-    if (n < 3000000) return 1;
-    return (int)std::max<size_t>(2, (n + 2000000) / 4000000);
+    return o.shards > 0 ? o.shards : 1;
 }
 
 cd_status screen_sharded(Call& C, const cd_elements* el, size_t n, double t0, double t1, double dt,
