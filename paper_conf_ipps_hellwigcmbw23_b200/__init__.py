@@ -357,17 +357,31 @@ def screen(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
     opt.stats = C.pointer(st)
     out = cd_conjunctions()
     _check(cd_screen_ex(E.s, E.n, float(t0), float(t1), float(dt), float(d), _mode(mode), opt, out))
-    try:
-        if opt.outputs_on_device:
-            raise ValueError("use screen_device() for device outputs")
-        if out.count:
-            buf = (C.c_char * (out.count * CONJ_DTYPE.itemsize)).from_address(out.data)
-            res = np.frombuffer(buf, dtype=CONJ_DTYPE).copy()
-        else:
-            res = np.zeros(0, dtype=CONJ_DTYPE)
-    finally:
+    if opt.outputs_on_device:
         cd_conjunctions_free(out)
+        raise ValueError("use cd_screen_ex with a device result for outputs_on_device")
+    if out.count:
+        # zero-copy view of the library-owned host result; released when the array is
+        buf = (C.c_char * (out.count * CONJ_DTYPE.itemsize)).from_address(out.data)
+        buf._owner = _ResultOwner(out)
+        res = np.frombuffer(buf, dtype=CONJ_DTYPE)
+    else:
+        cd_conjunctions_free(out)
+        res = np.zeros(0, dtype=CONJ_DTYPE)
     return (res, st.as_dict()) if return_stats else res
+
+
+class _ResultOwner:
+    """Frees a library-owned host result (cd_conjunctions_free) when the last view goes."""
+
+    def __init__(self, out):
+        self.out = out
+
+    def __del__(self):
+        try:
+            cd_conjunctions_free(self.out)
+        except Exception:
+            pass
 
 
 def candidates(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
