@@ -501,6 +501,13 @@ cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_opti
     const double* src[6] = {el->a, el->e, el->inc, el->raan, el->argp, el->nu0};
     if (o.inputs_on_device) {
         E = Elements{el->a, el->e, el->inc, el->raan, el->argp, el->nu0};
+    } else {
+        CU(up.alloc(6 * n));
+        for (int c = 0; c < 6; ++c)
+            CU(cudaMemcpyAsync(up.p + c * n, src[c], sizeof(double) * n, cudaMemcpyHostToDevice, st));
+        E = Elements{up.p, up.p + n, up.p + 2 * n, up.p + 3 * n, up.p + 4 * n, up.p + 5 * n};
+    }
+    {   // validation on the device (a > 0, 0 <= e < 1, finite angles): first bad index
         DBuf<int> bad(st);
         CU(bad.alloc(1));
         int init = 0x7fffffff;
@@ -512,12 +519,6 @@ cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_opti
         CU(cudaMemcpyAsync(&hb, bad.p, sizeof(int), cudaMemcpyDeviceToHost, st));
         CU(cudaStreamSynchronize(st));
         if (hb != 0x7fffffff) return fail(CD_EINVAL, "element %d: invalid (need a > 0, 0 <= e < 1, finite)", hb);
-    } else {
-        TRY(validate_elements_host(src, n));
-        CU(up.alloc(6 * n));
-        for (int c = 0; c < 6; ++c)
-            CU(cudaMemcpyAsync(up.p + c * n, src[c], sizeof(double) * n, cudaMemcpyHostToDevice, st));
-        E = Elements{up.p, up.p + n, up.p + 2 * n, up.p + 3 * n, up.p + 4 * n, up.p + 5 * n};
     }
     C.pt.start(kPhPrecompute);
     DBuf<uint32_t> key(st), idx(st), keyo(st);
