@@ -582,6 +582,23 @@ void orc_pair_distance(const orc_elements* el, int64_t i, int64_t j, const doubl
     }
 }
 
+/* R#14 test of one pair at time t: 1 iff |v_i - v_j| < 1e-9 km/s (D stationary); *D = D(t). */
+int orc_pair_degenerate(const orc_elements* el, int64_t i, int64_t j, double t, double* D)
+{
+    orc_orbit A, B;
+    orc_make_orbit(el, i, &A);
+    orc_make_orbit(el, j, &B);
+    double ra[3], va[3], rb[3], vb[3], dv2 = 0.0, dr2 = 0.0;
+    orc_state(&A, t, ra, va);
+    orc_state(&B, t, rb, vb);
+    for (int q = 0; q < 3; ++q) {
+        dv2 += (va[q] - vb[q]) * (va[q] - vb[q]);
+        dr2 += (ra[q] - rb[q]) * (ra[q] - rb[q]);
+    }
+    if (D) *D = sqrt(dr2);
+    return sqrt(dv2) < 1e-9;
+}
+
 void orc_free(void* p) { free(p); }
 
 /* Flags of arbitrary candidates (test helper for parity exclusions): ORC_MULTI when g changes

@@ -44,6 +44,7 @@ int64_t orc_conjunctions(const orc_elements* el, int64_t n, double t0, double t1
                          orc_conjunction** out);
 void    orc_pair_distance(const orc_elements* el, int64_t i, int64_t j, const double* t, int64_t nt,
                           double* D, double* g);
+int     orc_pair_degenerate(const orc_elements* el, int64_t i, int64_t j, double t, double* D);
 void    orc_candidate_flags(const orc_elements* el, int64_t n, double t0, double dt, double gc,
                             const orc_candidate* cand, int64_t ncand, uint32_t* flags);
 int     orc_pair_filter(const orc_elements* el, int64_t i, int64_t j, double d, double tlo,

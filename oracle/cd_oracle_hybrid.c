@@ -23,7 +23,9 @@
  *
  * Conjunctions: the local minima of D below d inside the intervals (sign changes of
  * g = dr.dv, 32 samples per interval, bisection to 1e-10 s), TCA in the owner cell.  Because
- * the filters are conservative the final set equals level O3 on the coarse candidates.
+ * the filters are conservative the final set equals level O3 on the coarse candidates --
+ * including O3's degenerate rows (R#14), which the coplanar path reports as O3 does (twins are
+ * coplanar: D = 0).
  */
 #include <math.h>
 #include <stdint.h>
@@ -256,8 +258,9 @@ int64_t orc_hybrid(const orc_elements* el, int64_t n, double t0, double t1, doub
         for (int64_t qd = 0; qd < nc; ++qd) {
             const orc_candidate* c = &cand[qd];
             double tk = fma((double)c->step, dt, t0);
+            /* owner cell; a single instant when t1 == t0, where only a degenerate coplanar
+             * pair has a row (R#14, as in O3) and the minima searches below find nothing */
             double oa = fmax(tk - 0.5 * dt, t0), ob = fmin(tk + 0.5 * dt, t1);
-            if (!(ob > oa)) continue;
             hy_orbit A, B;
             hy_make(el, c->i, &A);
             hy_make(el, c->j, &B);
@@ -273,7 +276,20 @@ int64_t orc_hybrid(const orc_elements* el, int64_t n, double t0, double t1, doub
             if (fl == ORC_H_COPLANAR) {
                 ls[1]++;
                 flags = ORC_COPLANAR;
-                m = hy_minima(el, c->i, c->j, oa, ob, oa, ob, d, tca, pca, 8);
+                /* "the procedure is the same as for the grid-based variant", so a
+                 * degenerate pair (D stationary) is reported as there: tca = t_k, pca = D(t_k)
+                 * (reading R#14) */
+                double Dk;
+                if (orc_pair_degenerate(el, c->i, c->j, tk, &Dk)) {
+                    if (Dk < d) {
+                        flags |= ORC_DEGENERATE;
+                        tca[0] = tk;
+                        pca[0] = Dk;
+                        m = 1;
+                    }
+                } else {
+                    m = hy_minima(el, c->i, c->j, oa, ob, oa, ob, d, tca, pca, 8);
+                }
             } else {
                 ls[4]++;
                 for (int w = 0; w < niv && m < 8; ++w)

@@ -19,3 +19,22 @@ def orc():
     import oracle
     oracle.lib()
     return oracle
+
+
+def pytest_terminal_summary(terminalreporter):
+    """Totals of the parity comparisons run this session: rows matched element by element and
+    rows set aside by the parity rules' exclusions (threshold/owner-boundary/MULTI), per kind."""
+    par = sys.modules.get("tests.parity") or sys.modules.get("parity")
+    if par is None or not getattr(par, "TALLY", None):
+        return
+    tot = {}
+    for kind, m, e in par.TALLY:
+        a = tot.setdefault(kind, [0, 0, 0])
+        a[0] += 1
+        a[1] += m
+        a[2] += e
+    terminalreporter.write_line("parity exclusions: " + "; ".join(
+        f"{k}: {c} comparisons, {m} matched, {e} excluded ({e / max(1, m + e):.2e})"
+        for k, (c, m, e) in sorted(tot.items())))
+    for (test, why), c in sorted(getattr(par, "REASONS", {}).items()):
+        terminalreporter.write_line(f"  excluded conjunctions, {why}: {c}  ({test})")

@@ -4,11 +4,13 @@
   1 mm of g_c (either side);
 * conjunctions: identical (i, j, step) sets excluding rows with |PCA - d| < 1 mm, TCA within
   1e-3 s of an owner-cell boundary t_k +- dt/2 or of t0 / t1, or the oracle's MULTI flag; matched
-  rows need |dTCA| <= 1e-3 s and |dPCA| <= 1 m.
+  rows need |dTCA| <= 1e-3 s and |dPCA| <= 1 m.  Stricter than SURVEY's rule: the PCA and TCA
+  exclusions apply only to a row one side lacks; a row on both sides is always compared.
 """
 from __future__ import annotations
 
 import math
+import os
 from collections import defaultdict
 
 import numpy as np
@@ -18,6 +20,16 @@ import oracle
 MM = 1e-6          # 1 mm in km
 TCA_TOL = 1e-3     # s
 PCA_TOL = 1e-3     # km (1 m)
+
+# Every comparison of the session adds (kind, matched, excluded) here; conftest.py prints the
+# totals, so the share of rows the parity rules exclude ("should be ~0") is visible
+# in every GPU run instead of being silently absorbed.
+TALLY: list[tuple[str, int, int]] = []
+REASONS: dict = defaultdict(int)       # (test, reason) -> excluded conjunction rows
+
+
+def _test_name():
+    return os.environ.get("PYTEST_CURRENT_TEST", "?").split(" ")[0]
 
 
 def _keys(a):
@@ -35,6 +47,7 @@ def compare_candidates(pop, gpu, orc, t0, dt, gc):
                                      f"{'gpu' if (i, j, k) in g else 'oracle'}: D = {D[0]!r}, "
                                      f"g_c = {gc}")
     assert len(gpu) == len(g), "duplicate candidates in the GPU output"
+    TALLY.append(("candidates", len(g & o), len(diff)))
     return len(diff)
 
 
@@ -63,11 +76,24 @@ def compare_conjunctions(pop, gpu, orc, t0, t1, dt, d, gc):
     if len(keys):
         ca["i"], ca["j"], ca["step"] = cand[:, 0], cand[:, 1], cand[:, 2]
     flags = dict(zip(keys, oracle.candidate_flags(pop, t0, dt, gc, ca).tolist())) if len(keys) else {}
-    matched = excluded = 0
+    matched = excluded = one_sided = 0
     for k in keys:
         g, o = G.get(k, []), O.get(k, [])
-        if flags[k] & oracle.MULTI or any(_excluded_row(r, t0, t1, dt, d) for r in g + o):
+        # the threshold / edge exclusions only excuse a row missing on one side: a row both
+        # sides report is compared whatever its TCA and PCA (only MULTI is set aside)
+        two_sided = len(g) == 1 and len(o) == 1
+        if flags[k] & oracle.MULTI or (not two_sided and any(_excluded_row(r, t0, t1, dt, d) for r in g + o)):
             excluded += 1
+            why = "multi" if flags[k] & oracle.MULTI else (
+                "pca~d" if any(abs(r["pca"] - d) < MM for r in g + o) else "tca~edge")
+            if len(g) == 1 and len(o) == 1:
+                agree = (abs(g[0]["tca"] - o[0]["tca"]) <= TCA_TOL
+                         and abs(g[0]["pca"] - o[0]["pca"]) <= PCA_TOL)
+                side = "both, agree" if agree else "both, differ"
+            else:
+                side = "gpu only" if g else "oracle only"
+                one_sided += 1
+            REASONS[(_test_name(), f"{why} [{side}]")] += 1
             continue
         assert len(g) == 1 and len(o) == 1, (k, g, o)
         g, o = g[0], o[0]
@@ -76,7 +102,8 @@ def compare_conjunctions(pop, gpu, orc, t0, t1, dt, d, gc):
         assert bool(g["flags"] & 2) == bool(o["flags"] & 2), (k, g, o)
         matched += 1
     assert len(gpu) == 0 or np.all(gpu["i"] < gpu["j"])
-    return {"matched": matched, "excluded": excluded}
+    TALLY.append(("conjunctions", matched, excluded))
+    return {"matched": matched, "excluded": excluded, "one_sided": one_sided}
 
 
 def is_sorted(a):
@@ -120,6 +147,7 @@ def compare_legacy(pop, gpu, orc, t0, t1, dt, d):
         assert abs(g["pca"] - o["pca"]) <= PCA_TOL, (k, g, o)
         assert (g["flags"] & 4) == (o["flags"] & 4), (k, g, o)
         matched += 1
+    TALLY.append(("legacy", matched, excluded))
     return {"matched": matched, "excluded": excluded}
 
 

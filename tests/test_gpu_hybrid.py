@@ -33,6 +33,18 @@ def _check(pop, t0, t1, dt, d, **kw):
     return res, st
 
 
+def test_hybrid_config1_full_window_with_twins():
+    """Config 1 (planted closed-form pairs, co-located twins, straddlers) over its whole 10-min
+    window at dt_h = 9 s: the twins take the coplanar path and come back DEGENERATE at every
+    coarse step on both sides (R14 via P:183); no row is one-sided."""
+    pop, cfg, _ = popgen.make_config(1)
+    res, _ = _check(pop, cfg.t0, cfg.t1, 9.0, cfg.d)
+    assert res["matched"] > 50 and res["one_sided"] == 0
+    Cg = cds.screen(pop, cfg.t0, cfg.t1, 9.0, cfg.d, mode="hybrid")
+    deg = Cg[(Cg["flags"] & cds.CD_FLAG_DEGENERATE) != 0]
+    assert len(deg) > 0 and np.all(deg["tca"] == cfg.t0 + deg["step"] * 9.0)
+
+
 def test_hybrid_catalog_30k():
     pop, cfg, _ = popgen.make_config(2)
     res, st = _check(pop, 0.0, 7200.0, 9.0, 2.0)

@@ -33,16 +33,38 @@ def test_conservative_against_unfiltered(orc):
     hyb, counts = orc.hybrid(pop, 0.0, 5400.0, dt, d)
     assert counts["candidates"] == len(K)
     assert counts["ap_rejected"] + counts["path_rejected"] + counts["time_rejected"] > 0.5 * len(K)
-    keep = (full["flags"] & orc.DEGENERATE) == 0
-    a = set(zip(full["i"][keep].tolist(), full["j"][keep].tolist(), full["step"][keep].tolist()))
+    _same_as_unfiltered(orc, full, hyb, min_rows=20)
+
+
+def _same_as_unfiltered(orc, full, hyb, min_rows):
+    a = set(zip(full["i"].tolist(), full["j"].tolist(), full["step"].tolist()))
     b = set(zip(hyb["i"].tolist(), hyb["j"].tolist(), hyb["step"].tolist()))
-    assert len(a) > 20
+    assert len(a) > min_rows
     assert a == b
-    # same minima (TCA, PCA) as the unfiltered search
-    fk = {(int(r["i"]), int(r["j"]), int(r["step"])): r for r in full[keep]}
+    # same minima (TCA, PCA) as the unfiltered search; degenerate rows (R14) on both sides
+    fk = {(int(r["i"]), int(r["j"]), int(r["step"])): r for r in full}
     for r in hyb:
         f = fk[(int(r["i"]), int(r["j"]), int(r["step"]))]
         assert abs(f["tca"] - r["tca"]) < 1e-6 and abs(f["pca"] - r["pca"]) < 1e-9
+        assert bool(f["flags"] & orc.DEGENERATE) == bool(r["flags"] & orc.DEGENERATE)
+
+
+def test_degenerate_twins_as_grid_variant(orc):
+    """Config 1's planted co-located twins: coplanar, so the hybrid refines them as the grid
+    variant does and reports them as O3 does (R14: tca = t_k, pca = D(t_k), DEGENERATE)
+    at every coarse step; every other row is O3's on the same coarse candidates."""
+    pop, cfg, _ = popgen.make_config(1)
+    dt, d = 9.0, cfg.d
+    gc = orc.cell_size(d, dt)
+    K = orc.candidates_grid(pop, cfg.t0, cfg.t1, dt, gc)
+    full = orc.conjunctions(pop, cfg.t0, cfg.t1, dt, d, gc, K)
+    hyb, counts = orc.hybrid(pop, cfg.t0, cfg.t1, dt, d)
+    deg = hyb[(hyb["flags"] & orc.DEGENERATE) != 0]
+    K_steps = orc.num_steps(cfg.t0, cfg.t1, dt)
+    assert len(deg) >= K_steps and len(deg) % K_steps == 0      # each twin pair at every step
+    assert np.all(deg["flags"] & orc.COPLANAR) and np.all(deg["pca"] < 1e-6)
+    assert np.all(deg["tca"] == cfg.t0 + deg["step"] * dt)
+    _same_as_unfiltered(orc, full, hyb, min_rows=K_steps)
 
 
 def test_ap_filter_disjoint_shells(orc):
