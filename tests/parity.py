@@ -134,14 +134,19 @@ def compare_legacy(pop, gpu, orc, t0, t1, dt, d):
     for k in sorted(set(G) | set(O)):
         g, o = G.get(k), O.get(k)
         rows = [r for r in (g, o) if r is not None]
-        if (o is not None and o["flags"] & MULTI_FLAG) or any(_excluded_row(r, t0, t1, dt, d) for r in rows):
+        multi = o is not None and bool(o["flags"] & MULTI_FLAG)
+        # as for the grid: threshold / edge exclusions only excuse a row one side lacks
+        if multi or (len(rows) == 1 and any(_excluded_row(r, t0, t1, dt, d) for r in rows)):
             excluded += 1
+            REASONS[(_test_name(), "legacy " + ("multi" if multi else "edge/threshold")
+                     + (" [both]" if len(rows) == 2 else " [one side]"))] += 1
             continue
         if g is None or o is None:
             tk = t0 + k[2] * dt
             n_min = _minima_near(pop, k[0], k[1], tk - 2 * dt, tk + 2 * dt, d)
             assert n_min >= 2, (k, g, o, n_min)
             excluded += 1
+            REASONS[(_test_name(), "legacy second minimum within 2 dt [one side]")] += 1
             continue
         assert abs(g["tca"] - o["tca"]) <= TCA_TOL, (k, g, o)
         assert abs(g["pca"] - o["pca"]) <= PCA_TOL, (k, g, o)
