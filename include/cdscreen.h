@@ -31,6 +31,16 @@
  *              CD_ECUDA with the driver's message.
  *   Threads    calls may be made from several host threads; each call uses its own stream and
  *              scratch memory.
+ *   Streams    a call runs on cd_options.stream when given: device-resident inputs must be
+ *              complete in that stream's order (e.g. written earlier on it), and device results
+ *              are ready in its order when the call returns.  Without one the library runs on a
+ *              stream of its own created blocking (cudaStreamDefault), so it is ordered after all
+ *              work queued earlier on the legacy default stream.  With cd_options.alloc, the
+ *              allocator's blocks are used on that same stream only.
+ *   Memory     device scratch comes from cd_options.alloc when given, else from a private
+ *              stream-ordered pool per device (the device's default pool is not touched) that
+ *              keeps its memory between calls; a per-device cache keeps the largest result
+ *              accumulation buffer (<= 1 GiB) between calls.  cd_release_caches() returns both.
  */
 #ifndef CDSCREEN_H
 #define CDSCREEN_H
@@ -42,7 +52,7 @@
 extern "C" {
 #endif
 
-#define CD_ABI_VERSION 2   /* 2: cd_options.propagator */
+#define CD_ABI_VERSION 3   /* 2: cd_options.propagator; 3: kepler_points honoured, cd_release_caches */
 
 typedef enum {
     CD_OK = 0,
@@ -50,7 +60,8 @@ typedef enum {
     CD_ENOMEM = 2,    /* device or host allocation failed even after capacity retries         */
     CD_ECUDA = 3,     /* a CUDA runtime/driver error; cd_last_error() has the message          */
     CD_ENCCL = 4,     /* reserved: collective failure (the merge runs in the Python layer)     */
-    CD_ERANGE = 5,    /* a position fell outside the key range +-(2^20 - 2) cells of g_c       */
+    CD_ERANGE = 5,    /* a position fell outside the key range +-(2^20 - 2) cells of the cell
+                         edge L >= g_c per axis (>= +-104,857 km at g_c = 0.1 km)              */
     CD_EINTERNAL = 6, /* internal invariant violated                                           */
     CD_ENODEV = 7     /* no CUDA device / the library was not built for this device            */
 } cd_status;
@@ -149,7 +160,10 @@ typedef struct {
                                  default 0, 1                                                 */
     int inputs_on_device;     /* element pointers are device pointers                         */
     int outputs_on_device;    /* cd_conjunctions.data stays in device memory                  */
-    int kepler_points;        /* 0 = choose the Contour point count per object from e         */
+    int kepler_points;        /* minimum Contour point count N (ref. [43]): 0 = per object
+                                 from e (4 for e <= 0.01, 6 <= 0.1, 8 <= 0.3, 12 <= 0.6, 16 above;
+                                 DESIGN.md R15); 4, 6, 8, 12 or 16 = at least that many points for
+                                 every object (more accuracy, more fp64 work); else CD_EINVAL    */
     double cell_factor;       /* grid cell edge = cell_factor * g_c (>= 1); 1 = the paper's cell
                                  and 27-cell scan; default 0 = auto (chosen from the measured
                                  candidate density; results do not depend on it)               */
@@ -266,6 +280,11 @@ cd_status cd_plan(size_t n, double t0, double t1, double dt, double d, cd_mode m
 cd_status cd_shell_members(const cd_elements* el, size_t n, double shell_lo, double shell_hi,
                            double gc, uint32_t* idx, size_t* count);
 void cd_candidates_free(cd_candidate* c);
+/* Release the library's cached device memory of `device` (-1: every device used so far): trim
+ * its private stream-ordered pool to zero (after a device synchronisation) and free the cached
+ * result accumulation buffer.  Results still held by the caller stay valid.  CD_EINVAL for a
+ * device out of range; CD_OK without any device. */
+cd_status cd_release_caches(int device);
 const char* cd_status_str(cd_status s);
 const char* cd_last_error(void);
 int cd_abi_version(void);

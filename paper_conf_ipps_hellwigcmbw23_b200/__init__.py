@@ -35,7 +35,9 @@ CAND_DTYPE = np.dtype([("i", "<u4"), ("j", "<u4"), ("step", "<u4")])
 # C ABI symbols declared in include/cdscreen.h
 ABI_SYMBOLS = ("cd_options_init", "cd_screen", "cd_screen_ex", "cd_candidates", "cd_propagate",
                "cd_conjunctions_sort_device", "cd_conjunctions_free", "cd_candidates_free", "cd_status_str", "cd_last_error",
-               "cd_abi_version", "cd_kernel_launches", "cd_plan", "cd_shell_members")
+               "cd_abi_version", "cd_kernel_launches", "cd_plan", "cd_shell_members",
+               "cd_release_caches")
+ABI_VERSION = 3
 
 
 class CdError(RuntimeError):
@@ -149,6 +151,10 @@ def lib():
         L.cd_plan.restype = C.c_int
         L.cd_plan.argtypes = [C.c_size_t, C.c_double, C.c_double, C.c_double, C.c_double, C.c_int,
                               C.c_size_t, P(cd_plan_info)]
+        L.cd_release_caches.restype = C.c_int
+        L.cd_release_caches.argtypes = [C.c_int]
+        if L.cd_abi_version() != ABI_VERSION:
+            raise ImportError(f"{LIB_PATH}: ABI {L.cd_abi_version()} != {ABI_VERSION}: rebuild it")
         _lib = L
     return _lib
 
@@ -219,24 +225,52 @@ def cd_plan(n, t0, t1, dt, d, mode, mem_bytes, out):
     return lib().cd_plan(n, t0, t1, dt, d, mode, mem_bytes, C.byref(out))
 
 
+def cd_release_caches(device=-1):
+    return lib().cd_release_caches(int(device))
+
+
 # numpy / torch wrappers --------------------------------------------------------------------
 class _Elements:
     """Holds the arrays alive while the C call runs.  numpy -> host pointers; torch CUDA
-    tensors -> device pointers (inputs_on_device)."""
+    tensors -> device pointers (inputs_on_device).  Validates the layout the C ABI assumes
+    (cdscreen.h cd_elements: six 1-D fp64 arrays of one length, all on one device) and raises
+    ValueError before any pointer reaches C."""
 
     def __init__(self, pop):
         # optional force model carried by the population dict ("kepler" / "j2")
         self.propagator = pop.get("propagator") if hasattr(pop, "get") else None
-        first = pop["a"]
-        self.on_device = hasattr(first, "is_cuda") and bool(first.is_cuda)
+        vals = [pop[k] for k in FIELDS]
+        cuda = [hasattr(v, "is_cuda") and bool(v.is_cuda) for v in vals]
+        if any(cuda) and not all(cuda):
+            raise ValueError("elements: mix of CUDA tensors and host arrays")
+        self.on_device = all(cuda)
+        self.device = None
         if self.on_device:
-            self.keep = [pop[k].contiguous() for k in FIELDS]
+            import torch
+            for k, v in zip(FIELDS, vals):
+                if v.dtype != torch.float64:
+                    raise ValueError(f"elements[{k!r}]: dtype {v.dtype}, need torch.float64")
+                if v.dim() != 1:
+                    raise ValueError(f"elements[{k!r}]: need a 1-D tensor, got shape {tuple(v.shape)}")
+            devs = {v.device.index for v in vals}
+            if len(devs) != 1:
+                raise ValueError(f"elements on several devices: {sorted(devs)}")
+            self.device = devs.pop()
+            self.keep = [v.contiguous() for v in vals]
             ptrs = [t.data_ptr() for t in self.keep]
-            self.n = int(self.keep[0].numel())
+            lens = [int(t.numel()) for t in self.keep]
         else:
-            self.keep = [np.ascontiguousarray(np.asarray(pop[k], dtype=np.float64)) for k in FIELDS]
+            self.keep = []
+            for k, v in zip(FIELDS, vals):
+                a = np.asarray(v)
+                if a.ndim != 1:
+                    raise ValueError(f"elements[{k!r}]: need a 1-D array, got shape {a.shape}")
+                self.keep.append(np.ascontiguousarray(a, dtype=np.float64))
             ptrs = [a.ctypes.data for a in self.keep]
-            self.n = int(self.keep[0].shape[0])
+            lens = [int(a.shape[0]) for a in self.keep]
+        if len(set(lens)) != 1:
+            raise ValueError(f"elements: arrays of different lengths {dict(zip(FIELDS, lens))}")
+        self.n = lens[0]
         self.s = cd_elements(*ptrs)
 
 
@@ -280,7 +314,7 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
                  cell_factor=None, batch_object_steps=None, round_steps=None,
                  outputs_on_device=False, inputs_on_device=False, profile_phases=False,
                  l2_persist=None, grid_table=None, propagator=None, shell=None, allocator=None,
-                 shards=None):
+                 shards=None, kepler_points=None):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -311,9 +345,18 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
     if shell is not None:
         o.shell_lo, o.shell_hi = float(shell[0]), float(shell[1])
     if allocator is not None:
+        # the allocator's blocks are stream-ordered on its stream: the call must run there
+        if stream is not None and int(stream or 0) != int(allocator.stream or 0):
+            raise ValueError("allocator and stream disagree: the call must run on the allocator's stream")
+        o.stream = allocator.stream
+        if device is not None and int(device) != allocator.device:
+            raise ValueError("allocator and device disagree")
+        o.device = allocator.device
         allocator.install(o)
     if shards is not None:
         o.shards = int(shards)
+    if kepler_points is not None:
+        o.kepler_points = int(kepler_points)
     return o
 
 
@@ -323,11 +366,11 @@ def _mode(mode):
     return int(mode)
 
 
-def _torch_stream():
+def _torch_stream(device=None):
     try:
         import torch
         if torch.cuda.is_available():
-            return torch.cuda.current_stream().cuda_stream
+            return torch.cuda.current_stream(device).cuda_stream
     except Exception:
         pass
     return None
@@ -345,15 +388,26 @@ def _resolve_allocator(kw):
     return kw.get("allocator")
 
 
+def _device_options(E, kw):
+    """Device inputs (CUDA tensors): run on their device and, unless a stream is given, on torch's
+    current stream there -- the stream that wrote them (cdscreen.h "Streams")."""
+    if not E.on_device:
+        return
+    if kw.get("device") is not None and int(kw["device"]) != E.device:
+        raise ValueError(f"device={kw['device']} but the elements live on cuda:{E.device}")
+    kw["device"] = E.device
+    if kw.get("stream") is None and kw.get("allocator") is None:
+        kw["stream"] = _torch_stream(E.device)
+
+
 def screen(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
     """Conjunctions as a structured numpy array (CONJ_DTYPE), sorted by (i, j, step)."""
     E = _Elements(pop)
     st = cd_stats()
     kw.setdefault("propagator", E.propagator)
     keep_alloc = _resolve_allocator(kw)   # noqa: F841 (alive for the call)
+    _device_options(E, kw)
     opt = make_options(inputs_on_device=E.on_device, **kw)
-    if opt.stream is None and E.on_device:
-        opt.stream = _torch_stream()
     opt.stats = C.pointer(st)
     out = cd_conjunctions()
     _check(cd_screen_ex(E.s, E.n, float(t0), float(t1), float(dt), float(d), _mode(mode), opt, out))
@@ -390,6 +444,7 @@ def candidates(pop, t0, t1, dt, d, mode="grid", return_stats=False, **kw):
     st = cd_stats()
     kw.setdefault("propagator", E.propagator)
     keep_alloc = _resolve_allocator(kw)   # noqa: F841
+    _device_options(E, kw)
     opt = make_options(inputs_on_device=E.on_device, **kw)
     opt.stats = C.pointer(st)
     p = C.c_void_p()
@@ -414,11 +469,17 @@ def propagate(pop, times, velocity=False, **kw):
     xyz = np.zeros((t.size, E.n, 3))
     v = np.zeros((t.size, E.n, 3)) if velocity else None
     kw.setdefault("propagator", E.propagator)
+    _device_options(E, kw)
     opt = make_options(inputs_on_device=E.on_device, **kw)
     _check(cd_propagate(E.s, E.n, t.ctypes.data, t.size, xyz.ctypes.data,
                         v.ctypes.data if velocity else None, opt))
     return (xyz, v) if velocity else xyz
 
+
+
+def release_caches(device=-1):
+    """Return the library's cached device memory (private pool, result buffer cache)."""
+    _check(cd_release_caches(device))
 
 
 def plan(n, t0, t1, dt, d, mode="grid", mem_bytes=0):

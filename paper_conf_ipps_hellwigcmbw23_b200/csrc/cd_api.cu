@@ -107,7 +107,7 @@ struct DBuf {
 };
 
 std::mutex g_pool_mu;
-bool g_pool_done[64] = {};
+cudaMemPool_t g_pools[64] = {};
 
 // Per-host-thread page-locked staging for the per-round counters (4 Ctrl-sized slots), allocated
 // once and kept for the thread's lifetime: no call pays cudaMallocHost / cudaFreeHost.
@@ -183,10 +183,12 @@ cudaError_t copy_to_pageable(void* dst, const void* src, size_t bytes, cudaStrea
     return e;
 }
 
-// Per-device cache of the (unsorted) conjunction accumulation buffer (cudaMalloc'd): grow-only, handed from
-// call to call so a repeated or long screen does not regrow it (growing a stream-ordered pool by
-// hundreds of MB is a blocking driver call that stalls the round pipeline for up to ~1 s).  The
-// event orders the next user after the last use (the finalize sort) on the previous call's stream.
+// Per-device cache of the (unsorted) conjunction accumulation buffer (cudaMalloc'd): grow-only up
+// to kConjCacheMax bytes, handed from call to call so a repeated or long screen does not regrow it
+// (growing a stream-ordered pool by hundreds of MB is a blocking driver call that stalls the round
+// pipeline for up to ~1 s).  The event orders the next user after the last use (the finalize sort)
+// on the previous call's stream.  cd_release_caches() frees it.
+constexpr size_t kConjCacheMax = size_t(1) << 30;
 struct ConjCache {
     std::mutex mu;
     Conj* p = nullptr;
@@ -220,7 +222,7 @@ void conj_cache_give(int dev, cudaStream_t st, Conj* p, size_t cap)
     }
     ConjCache& c = g_conj_cache[dev];
     std::lock_guard<std::mutex> lk(c.mu);
-    if (c.p && c.cap >= cap) {
+    if ((c.p && c.cap >= cap) || sizeof(Conj) * cap > kConjCacheMax) {
         cudaFree(p);
         return;
     }
@@ -240,16 +242,27 @@ void conj_cache_give(int dev, cudaStream_t st, Conj* p, size_t cap)
 // Compute capability per device, queried once (cudaGetDeviceProperties costs milliseconds).
 int g_cc[64];   // 0 = not yet queried, else major * 10 + minor
 
-void setup_pool(int dev)
+// The library's private stream-ordered pool of device dev (see cd_internal.h g_pool).
+cudaMemPool_t setup_pool(int dev)
 {
     std::lock_guard<std::mutex> lk(g_pool_mu);
-    if (dev < 0 || dev >= 64 || g_pool_done[dev]) return;
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    if (dev < 0 || dev >= 64) return nullptr;
+    if (!g_pools[dev]) {
+        cudaMemPoolProps props = {};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.handleTypes = cudaMemHandleTypeNone;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        cudaMemPool_t pool = nullptr;
+        if (cudaMemPoolCreate(&pool, &props) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;   // fall back to the device's current pool (cudaMallocAsync)
+        }
         uint64_t thr = ~uint64_t(0);
         cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+        g_pools[dev] = pool;
     }
-    g_pool_done[dev] = true;
+    return g_pools[dev];
 }
 
 struct Owner {
@@ -372,6 +385,7 @@ struct Call {
     ~Call()
     {
         g_dev_alloc = DevAlloc{};
+        g_pool = nullptr;
         if (ev0) cudaEventDestroy(ev0);
         if (ev1) cudaEventDestroy(ev1);
         if (own_stream && st) {
@@ -400,12 +414,14 @@ struct Call {
         if (cc != 100)
             return fail(CD_ENODEV, "libcdscreen is built for sm_100a (B200); device %d is sm_%d",
                         dev, cc);
-        setup_pool(dev);
+        g_pool = setup_pool(dev);
         g_dev_alloc = DevAlloc{o.alloc, o.free, o.alloc_ctx};
         if (o.stream) {
             st = (cudaStream_t)o.stream;
         } else {
-            CU(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+            // a blocking stream: ordered after the work already queued on the legacy default
+            // stream (e.g. the copies that produced device-resident inputs), cdscreen.h "Streams"
+            CU(cudaStreamCreateWithFlags(&st, cudaStreamDefault));
             own_stream = true;
         }
         CU(cudaEventCreate(&ev0));
@@ -435,6 +451,8 @@ cd_status validate_scalars(size_t n, double t0, double t1, double dt, double d, 
     if (o.propagator != CD_PROP_KEPLER && o.propagator != CD_PROP_J2)
         return fail(CD_EINVAL, "unknown propagator %d", o.propagator);
     if (o.shards < 0 || o.shards > 64) return fail(CD_EINVAL, "need 0 <= shards <= 64");
+    if (kepler_class_of_points(o.kepler_points) < 0)
+        return fail(CD_EINVAL, "kepler_points = %d: need 0 (per e) or 4, 6, 8, 12, 16", o.kepler_points);
     if ((o.alloc == nullptr) != (o.free == nullptr))
         return fail(CD_EINVAL, "cd_options.alloc and free must be given together");
     if (!is_fin(o.shell_lo) || !is_fin(o.shell_hi) || o.shell_lo < 0.0 ||
@@ -529,14 +547,15 @@ cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_opti
     DBuf<unsigned long long> n0(st);
     CU(n0.alloc(1));
     CU(cudaMemsetAsync(n0.p, 0, sizeof(unsigned long long), st));
-    CU(launch_classify(E, (int64_t)n, key.p, idx.p, n0.p, st, C.lc));
+    const int min_cls = kepler_class_of_points(o.kepler_points);
+    CU(launch_classify(E, (int64_t)n, key.p, idx.p, n0.p, min_cls, st, C.lc));
     unsigned long long hn0 = 0;
     CU(cudaMemcpyAsync(&hn0, n0.p, sizeof hn0, cudaMemcpyDeviceToHost, st));
     CU(sort_pairs_u32(key.p, keyo.p, idx.p, S.perm.p, n, 3, st, C.lc));
     S.j2 = o.propagator == CD_PROP_J2;
     CU(S.rec.alloc((size_t)(S.j2 ? kNCol : kDOm) * n));   // the J2 columns only when used
     CU(S.cls.alloc(n));
-    CU(launch_build_records(E, S.perm.p, (int64_t)n, S.rec.p, S.cls.p, S.j2, st, C.lc));
+    CU(launch_build_records(E, S.perm.p, (int64_t)n, S.rec.p, S.cls.p, S.j2, min_cls, st, C.lc));
     C.pt.stop();
     CU(cudaStreamSynchronize(st));   // hn0 is needed on the host
     S.n0 = (int64_t)hn0;
@@ -972,7 +991,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         if (hctrl->err_internal)
             return fail(CD_EINTERNAL, "internal: a grid cell list did not terminate");
         if (hctrl->err_range)
-            return fail(CD_ERANGE, "a position fell outside the cell-key range (+-%lld cells of %g km)",
+            return fail(CD_ERANGE, "a position fell outside the cell-key range (+-%lld cells of edge %g km)",
                         (long long)kCellMax, L);
         bool redo = false;
         if (hctrl->n_cand > rd.qcap) {
@@ -1513,6 +1532,10 @@ cd_status cd_propagate(const cd_elements* el, size_t n, const double* t, size_t 
         for (size_t q = 0; q < nt; ++q)
             if (!is_fin(t[q])) return fail(CD_EINVAL, "non-finite time");
         const cd_options o = opt ? *opt : defaults();
+        if (kepler_class_of_points(o.kepler_points) < 0)
+            return fail(CD_EINVAL, "kepler_points = %d: need 0 (per e) or 4, 6, 8, 12, 16", o.kepler_points);
+        if (o.propagator != CD_PROP_KEPLER && o.propagator != CD_PROP_J2)
+            return fail(CD_EINVAL, "unknown propagator %d", o.propagator);
         Call C;
         TRY(C.begin(o));
         OrbitSet S;
@@ -1608,7 +1631,7 @@ cd_status cd_plan(size_t n, double t0, double t1, double dt, double d, cd_mode m
         const double wcap = std::min(qcap, std::max(4194304.0, 4.0 * nn));
         out->fixed_bytes = 48.0 * nn + (8.0 * kDOm + 1.0 + 4.0) * nn + 12.0 * qcap + 24.0 * wcap;
         // a_gh + a_l of one step's grid, in the structure the auto cell edge selects for the
-        // a-priori density: chained heads (4 B x next_pow2(4n)) in ball mode, the open map
+        // a-priori density: chained heads (4 B x next_pow2(8n)) in ball mode, the open map
         // (16 B x next_pow2(2n) slots + next_pow2(32n)-bit occupancy) in half-shell mode, plus the
         // 32-byte entries {x, y, z, next}
         const double m = choose_cell_factor(std::max(1.0, out->est_candidates_per_step) / std::max(1.0, nn));
@@ -1627,6 +1650,43 @@ cd_status cd_plan(size_t n, double t0, double t1, double dt, double d, cd_mode m
 }
 
 void cd_candidates_free(cd_candidate* c) { free(c); }
+
+cd_status cd_release_caches(int device)
+{
+    try {
+        int ndev = 0;
+        if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+            cudaGetLastError();
+            return CD_OK;   // nothing was ever cached
+        }
+        int prev = 0;
+        CU(cudaGetDevice(&prev));
+        const int lo = device >= 0 ? device : 0, hi = device >= 0 ? device + 1 : std::min(ndev, 64);
+        if (device >= ndev) return fail(CD_EINVAL, "device %d out of range (%d devices)", device, ndev);
+        for (int dv = lo; dv < hi; ++dv) {
+            CU(cudaSetDevice(dv));
+            {
+                ConjCache& c = g_conj_cache[dv];
+                std::lock_guard<std::mutex> lk(c.mu);
+                if (c.p) {
+                    if (c.ready) cudaEventSynchronize(c.ready);
+                    cudaFree(c.p);
+                }
+                c.p = nullptr;
+                c.cap = 0;
+            }
+            std::lock_guard<std::mutex> lk(g_pool_mu);
+            if (g_pools[dv]) {
+                CU(cudaDeviceSynchronize());   // blocks freed stream-ordered are back in the pool
+                CU(cudaMemPoolTrimTo(g_pools[dv], 0));
+            }
+        }
+        CU(cudaSetDevice(prev));
+        return CD_OK;
+    } catch (...) {
+        return fail(CD_EINTERNAL, "unexpected C++ exception");
+    }
+}
 
 const char* cd_status_str(cd_status s)
 {

@@ -47,6 +47,12 @@ __host__ __device__ inline int ecc_class(double e)
 {
     return e <= 0.01 ? 0 : e <= 0.1 ? 1 : e <= 0.3 ? 2 : e <= 0.6 ? 3 : 4;
 }
+// class of a requested point count (cd_options.kepler_points): 0 -> 0 (per e), 4/6/8/12/16 ->
+// class 0..4, anything else -> -1 (invalid)
+__host__ __device__ inline int kepler_class_of_points(int pts)
+{
+    return pts == 0 || pts == 4 ? 0 : pts == 6 ? 1 : pts == 8 ? 2 : pts == 12 ? 3 : pts == 16 ? 4 : -1;
+}
 
 struct Orbits {
     const double* rec;   // kNCol x n
@@ -370,21 +376,21 @@ __device__ __forceinline__ void state(const Orbits& O, int64_t r, double t, doub
 // ---------------------------------------------------------------------------------------
 // grid cells and keys ("calculates the grid cell based on the Cartesian coordinates")
 // ---------------------------------------------------------------------------------------
-// Cell keys pack 19 bits per axis (cells in [-(2^18 - 2), 2^18 - 2], i.e. +-262,142 cells of
-// edge L >= g_c: +-46,000 km at g_c = 0.18 km); the top 7 bits of a stored key word hold the tag
-// (1..126) of the build pass that wrote it.  A slot whose tag differs from the current pass is
-// empty (P:147 reserves a value for "empty"; tagging lets a table be reused without clearing it
-// every step -- tables are zeroed only when the tags wrap).
-constexpr int64_t kKeyBias = int64_t(1) << 18;
+// Cell keys pack 21 bits per axis: cells in [-(2^20 - 2), 2^20 - 2], i.e.
+// +-1,048,574 cells of edge L >= g_c -- +-104,857 km at g_c = 0.1 km, beyond GEO for any g_c >=
+// 0.05 km (P:128's (85,000 km)^3 space).  Bit 63 is 0.  The open map keeps the tag of the build
+// pass that wrote a slot (1..kMaxTag) in the upper half of the slot's head word: a slot whose tag
+// differs from the current pass is empty (P:147 reserves a value for "empty"; tagging lets a
+// table be reused without clearing it every step -- tables are zeroed only when the tags wrap).
+constexpr int64_t kKeyBias = int64_t(1) << 20;
 constexpr int64_t kCellMax = kKeyBias - 2;   // valid cells in [-kCellMax, kCellMax]
-constexpr int kTagShift = 57;
-constexpr uint32_t kMaxTag = 126;
+constexpr uint32_t kMaxTag = 0x7ffffffeu;
 constexpr uint32_t kNil = 0xffffffffu;
 
 __device__ __forceinline__ uint64_t pack_key(int cx, int cy, int cz)
 {
-    return uint64_t(uint32_t(cx + (int)kKeyBias)) | (uint64_t(uint32_t(cy + (int)kKeyBias)) << 19) |
-           (uint64_t(uint32_t(cz + (int)kKeyBias)) << 38);
+    return uint64_t(uint32_t(cx + (int)kKeyBias)) | (uint64_t(uint32_t(cy + (int)kKeyBias)) << 21) |
+           (uint64_t(uint32_t(cz + (int)kKeyBias)) << 42);
 }
 
 // MurmurHash3 64-bit finaliser (footnote 3: smhasher)
@@ -475,13 +481,13 @@ struct __align__(32) Entry {
 
 // Hash grid of one step.  Open addressing over M = 2^m >= 2n slots,
 // linear probing s_{i+1} = s_i + 1 mod M (Eq. 2) from the MurmurHash3 slot.  A slot is
-// 16 bytes {cell key | tag, list head}: key and head are installed together by one 128-bit CAS
-// (P:147-148's CAS, widened so that claiming a cell and pushing the first object onto its list is
-// a single atomic).  An all-zero slot is empty (P:147 reserves one value for "empty"; zero lets
-// tables be cleared with plain coalesced stores); keys carry a non-zero tag in their top bits.
+// 16 bytes {cell key, tag << 32 | list head}: key and head are installed together by one 128-bit
+// CAS (P:147-148's CAS, widened so that claiming a cell and pushing the first object onto its
+// list is a single atomic).  A slot whose tag is not the current pass's is empty (an all-zero
+// slot has tag 0, never used: tables are cleared with plain coalesced stores).
 struct __align__(16) Slot {
-    unsigned long long key;    // pack_key(cell) | tag << 57
-    unsigned long long head;   // low 32 bits: entry index of the list head (Fig. 6)
+    unsigned long long key;    // pack_key(cell)
+    unsigned long long head;   // tag << 32 | entry index of the list head (Fig. 6)
 };
 
 __device__ __forceinline__ bool cas128(Slot* s, unsigned long long& e0, unsigned long long& e1,
@@ -502,24 +508,24 @@ __device__ __forceinline__ bool cas128(Slot* s, unsigned long long& e0, unsigned
     return ok;
 }
 
-// Non-blocking insert of object r into the cell `key`.  A slot whose key word carries
-// another pass's tag is empty: it is claimed by a 128-bit CAS against the value just read; a slot
-// already holding the key (this pass) pushes r onto its list (CAS of the head); a slot of another
-// cell moves on along the probe sequence (Eq. 2).  Returns the previous list head (r's `next`),
-// kNil if r is the first object of its cell.
+// Non-blocking insert of object r into the cell `key`.  A slot carrying another
+// pass's tag is empty: it is claimed by a 128-bit CAS against the value just read; a slot already
+// holding the key (this pass) pushes r onto its list (CAS of the head word); a slot of another cell
+// moves on along the probe sequence (Eq. 2).  Returns the previous list head (r's `next`), kNil if
+// r is the first object of its cell.
 __device__ __forceinline__ uint32_t grid_insert(Slot* slots, uint64_t mask, unsigned long long key,
                                                 uint32_t tag, uint32_t r)
 {
-    const unsigned long long tk = key | ((unsigned long long)tag << kTagShift);
+    const unsigned long long th = (unsigned long long)tag << 32;
     uint64_t h = fmix64(key) & mask;
     while (true) {
         unsigned long long w0, w1;
         asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(w0), "=l"(w1) : "l"(slots + h));
         while (true) {
-            const bool stale = (uint32_t)(w0 >> kTagShift) != tag;
-            if (!stale && w0 != tk) break;   // another cell of this pass: next slot
+            const bool stale = (uint32_t)(w1 >> 32) != tag;
+            if (!stale && w0 != key) break;   // another cell of this pass: next slot
             const unsigned long long prev = w1;
-            if (cas128(slots + h, w0, w1, tk, (unsigned long long)r))
+            if (cas128(slots + h, w0, w1, key, th | (unsigned long long)r))
                 return stale ? kNil : (uint32_t)prev;
             // lost a race: (w0, w1) now hold the slot's current contents; re-evaluate
         }
@@ -541,12 +547,11 @@ struct GridTab {
 __device__ __forceinline__ uint32_t grid_find(const Slot* __restrict__ slots, uint64_t mask,
                                               unsigned long long key, uint32_t tag)
 {
-    const unsigned long long tk = key | ((unsigned long long)tag << kTagShift);
     uint64_t h = fmix64(key) & mask;
     while (true) {
         const ulonglong2 w = __ldg(reinterpret_cast<const ulonglong2*>(slots + h));
-        if (w.x == tk) return (uint32_t)w.y;
-        if ((uint32_t)(w.x >> kTagShift) != tag) return kNil;
+        if ((uint32_t)(w.y >> 32) != tag) return kNil;   // empty: the cell is not in the table
+        if (w.x == key) return (uint32_t)w.y;
         h = (h + 1) & mask;
     }
 }

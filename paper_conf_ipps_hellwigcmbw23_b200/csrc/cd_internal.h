@@ -28,6 +28,12 @@ struct DevAlloc {
 };
 extern thread_local DevAlloc g_dev_alloc;
 
+// The library's own stream-ordered pool of the call's device (created on first use with
+// cudaMemPoolCreate; the device's default pool and its settings are left alone).  It keeps its
+// memory between calls (release threshold = max) so back-to-back screens do not re-map pages;
+// cd_release_caches() trims it.
+extern thread_local cudaMemPool_t g_pool;
+
 inline cudaError_t dev_malloc(void** p, size_t bytes, cudaStream_t st)
 {
     if (bytes == 0) bytes = 1;
@@ -35,6 +41,7 @@ inline cudaError_t dev_malloc(void** p, size_t bytes, cudaStream_t st)
         *p = g_dev_alloc.alloc(bytes, g_dev_alloc.ctx);
         return *p ? cudaSuccess : cudaErrorMemoryAllocation;
     }
+    if (g_pool) return cudaMallocFromPoolAsync(p, bytes, g_pool, st);
     return cudaMallocAsync(p, bytes, st);
 }
 
@@ -68,10 +75,13 @@ struct RefineParams {
 };
 
 // ---- precompute (a1) -------------------------------------------------------------------
+// min_cls: minimum eccentricity class (Contour point count) of every object, from
+// cd_options.kepler_points (kepler_class_of_points)
 cudaError_t launch_classify(const Elements& el, int64_t n, uint32_t* key, uint32_t* idx,
-                            unsigned long long* n0, cudaStream_t st, LaunchCount& lc);
+                            unsigned long long* n0, int min_cls, cudaStream_t st, LaunchCount& lc);
 cudaError_t launch_build_records(const Elements& el, const uint32_t* perm, int64_t n,
-                                 double* rec, uint8_t* cls, int j2, cudaStream_t st, LaunchCount& lc);
+                                 double* rec, uint8_t* cls, int j2, int min_cls, cudaStream_t st,
+                                 LaunchCount& lc);
 cudaError_t launch_propagate_out(const cdk::Orbits& O, const uint32_t* perm, const double* t,
                                  int64_t nt, double* xyz, double* vxyz, cudaStream_t st,
                                  LaunchCount& lc);
@@ -85,8 +95,6 @@ cudaError_t launch_conj_to_global(const cdk::Conj* in, size_t n, const uint32_t*
                                   cdk::Conj* out, cudaStream_t st, LaunchCount& lc);
 
 // ---- grid build + scan (a2-a6) ---------------------------------------------------------
-cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long long v,
-                            cudaStream_t st, LaunchCount& lc);
 // One batch launch of the fused step kernel: build batch b+1 into build_tab (slots tagged
 // build_tag, bitmap zero on entry), scan batch b in scan_tab (tag scan_tag), zero the bitmap set
 // zero_bits (zero_depth tables) for batch b+2.

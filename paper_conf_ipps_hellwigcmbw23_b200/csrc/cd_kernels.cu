@@ -17,6 +17,7 @@ namespace cdh {
 
 std::atomic<uint64_t> g_launches{0};
 thread_local DevAlloc g_dev_alloc;
+thread_local cudaMemPool_t g_pool = nullptr;
 
 static inline unsigned blocks_for(int64_t n, int t) { return (unsigned)((n + t - 1) / t); }
 
@@ -64,19 +65,21 @@ __device__ __forceinline__ void append_count(unsigned long long* cnt)
 // ---------------------------------------------------------------------------------------
 // a1: per-object precompute
 // ---------------------------------------------------------------------------------------
+// min_cls: the class of cd_options.kepler_points (0 = per e only); an object takes the larger of
+// its eccentricity class and min_cls, i.e. at least the requested Contour point count
 __global__ void k_classify(Elements el, int64_t n, uint32_t* key, uint32_t* idx,
-                           unsigned long long* n0)
+                           unsigned long long* n0, int min_cls)
 {
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i >= n) return;
-    const int cl = ecc_class(el.e[i]);
+    const int cl = max(ecc_class(el.e[i]), min_cls);
     key[i] = (uint32_t)cl;
     idx[i] = (uint32_t)i;
     if (cl == 0) append_count(n0);
 }
 
 __global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, int64_t n,
-                                double* __restrict__ rec, uint8_t* __restrict__ cls, int j2)
+                                double* __restrict__ rec, uint8_t* __restrict__ cls, int j2, int min_cls)
 {
     const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (r >= n) return;
@@ -122,7 +125,7 @@ __global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, 
     const double rho = 0.5 * e;
     put(kEcr, e * cos(rho));
     put(kEsr, e * sin(rho));
-    const int cl = ecc_class(e);
+    const int cl = max(ecc_class(e), min_cls);
     const int N = class_points(cl);
     for (int j = 1; j <= (N - 2) / 2; ++j) {
         const double ct = kNodes[cl][j - 1][0], st = kNodes[cl][j - 1][1];
@@ -152,17 +155,17 @@ __global__ void k_propagate_out(Orbits O, const uint32_t* __restrict__ perm,
 }
 
 cudaError_t launch_classify(const Elements& el, int64_t n, uint32_t* key, uint32_t* idx,
-                            unsigned long long* n0, cudaStream_t st, LaunchCount& lc)
+                            unsigned long long* n0, int min_cls, cudaStream_t st, LaunchCount& lc)
 {
-    k_classify<<<blocks_for(n, 256), 256, 0, st>>>(el, n, key, idx, n0);
+    k_classify<<<blocks_for(n, 256), 256, 0, st>>>(el, n, key, idx, n0, min_cls);
     lc.bump();
     return cudaGetLastError();
 }
 
 cudaError_t launch_build_records(const Elements& el, const uint32_t* perm, int64_t n, double* rec,
-                                 uint8_t* cls, int j2, cudaStream_t st, LaunchCount& lc)
+                                 uint8_t* cls, int j2, int min_cls, cudaStream_t st, LaunchCount& lc)
 {
-    k_build_records<<<blocks_for(n, 128), 128, 0, st>>>(el, perm, n, rec, cls, j2);
+    k_build_records<<<blocks_for(n, 128), 128, 0, st>>>(el, perm, n, rec, cls, j2, min_cls);
     lc.bump();
     return cudaGetLastError();
 }
@@ -243,28 +246,6 @@ cudaError_t launch_conj_to_global(const Conj* in, size_t n, const uint32_t* perm
 }
 
 // ---------------------------------------------------------------------------------------
-// a4 helper: clear hash tables to the empty marker ("initialized with this value")
-// ---------------------------------------------------------------------------------------
-__global__ void k_fill_u64(ulonglong2* __restrict__ p, size_t n2, unsigned long long v)
-{
-    const size_t stride = (size_t)gridDim.x * blockDim.x;
-    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n2; i += stride)
-        p[i] = make_ulonglong2(v, v);
-}
-
-cudaError_t launch_fill_u64(unsigned long long* p, size_t count, unsigned long long v,
-                            cudaStream_t st, LaunchCount& lc)
-{
-    const size_t n2 = count / 2;   // count is even (slots are 2 words)
-    unsigned blocks = (unsigned)((n2 + 255) / 256);
-    if (blocks > 148 * 16) blocks = 148 * 16;
-    if (blocks == 0) blocks = 1;
-    k_fill_u64<<<blocks, 256, 0, st>>>(reinterpret_cast<ulonglong2*>(p), n2, v);
-    lc.bump();
-    return cudaGetLastError();
-}
-
-// ---------------------------------------------------------------------------------------
 // a2-a4: build -- one thread per (object, step) ("one thread per tuple"): Contour Kepler
 // solve and Cartesian position, cell key, non-blocking insert into the step's hash grid
 // (Eq. 2) and its occupancy bitmap; the entry {x, y, z, next} (Fig. 6) is
@@ -277,11 +258,7 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
 {
     const double t = fma((double)(k0 + s), dt, t0);
     double p[3], v[3];
-#ifdef CD_ABL_NO_PROP   // ablation (timing experiments only): position from one record column
-    p[0] = O.at(kAPx, r) + t; p[1] = O.at(kAPy, r); p[2] = O.at(kAPz, r);
-#else
     state<false, kClass0 ? 0 : -1, kJ2>(O, r, t, p, v);
-#endif
     int c[3];
     uint32_t next = kNil, ctag = 0;
     if (kChained && cell_of(g, p, c)) {
@@ -289,24 +266,14 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
         // chained spatial hash: push onto the list of bucket hash(cell) -- one atomic exchange;
         // heads hold index + 1 (0 = empty bucket)
         const uint32_t b = chain_bucket(c[0], c[1], c[2], tab.bmask);
-#ifndef CD_ABL_NO_EXCH
         const uint32_t prev = atomicExch(tab.bits + (size_t)s * tab.bwords + b,
                                          (tag << kEpochShift) | ((uint32_t)r + 1u));
         next = ((prev >> kEpochShift) == tag && (prev & kIdxMask)) ? (prev & kIdxMask) - 1u : kNil;
-#else
-        next = b == 0xffffffffu ? 0u : kNil;
-#endif
     } else if (!kChained && cell_of(g, p, c)) {
         const unsigned long long key = pack_key(c[0], c[1], c[2]);
         const uint32_t hb = bit_hash(c[0], c[1], c[2]) & tab.bmask;
-#ifndef CD_ABL_NO_RED
         atomicOr(tab.bits + (size_t)s * tab.bwords + (hb >> 5), 1u << (hb & 31));
-#endif
-#ifndef CD_ABL_NO_CAS
         next = grid_insert(tab.slots + (size_t)s * (mask + 1), mask, key, tag, (uint32_t)r);
-#else
-        next = (uint32_t)(key & 0) | kNil;
-#endif
     } else {
         ctrl->err_range = 1;
     }
@@ -316,20 +283,7 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
     en.z = p[2];
     en.next = next;
     en.tag = ctag;
-#ifdef CD_STREAM_ENTRIES
-    // written once here, read once (coalesced) by the next launch's scan: stream past L2 so the
-    // randomly accessed slot table and bitmaps keep it
-    double4* dst = reinterpret_cast<double4*>(ents + (size_t)s * O.n + r);
-    double4 v4;
-    v4.x = en.x;
-    v4.y = en.y;
-    v4.z = en.z;
-    v4.w = __longlong_as_double((long long)en.next);
-    __stcs(reinterpret_cast<double2*>(dst), make_double2(v4.x, v4.y));
-    __stcs(reinterpret_cast<double2*>(dst) + 1, make_double2(v4.z, v4.w));
-#else
     ents[(size_t)s * O.n + r] = en;
-#endif
 }
 
 // ---------------------------------------------------------------------------------------
@@ -430,20 +384,7 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
     const uint32_t bmask = tab.bmask;
     const Entry* E = ents + (size_t)s * n;
     const uint32_t step = (uint32_t)(k0 + s);
-#ifdef CD_STREAM_ENTRIES
-    Entry me;
-    {
-        const double2 a = __ldcs(reinterpret_cast<const double2*>(E + r));
-        const double2 b = __ldcs(reinterpret_cast<const double2*>(E + r) + 1);
-        me.x = a.x;
-        me.y = a.y;
-        me.z = b.x;
-        me.next = (uint32_t)__double_as_longlong(b.y);
-        me.pad = 0;
-    }
-#else
     const Entry me = E[r];
-#endif
     const double p[3] = {me.x, me.y, me.z};
     int c[3];
     double fr[3];
@@ -474,7 +415,7 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
         const int d0 = fr[0] < rl ? -1 : (fr[0] > 1.0 - rl ? 1 : 0);
         const int d1 = fr[1] < rl ? -1 : (fr[1] > 1.0 - rl ? 1 : 0);
         const int d2 = fr[2] < rl ? -1 : (fr[2] > 1.0 - rl ? 1 : 0);
-        // (c +- 1 stays inside the 19-bit key range because |c| <= kCellMax = 2^18 - 2)
+        // (c +- 1 stays inside the 21-bit key range because |c| <= kCellMax = 2^20 - 2)
         const uint32_t hx1 = hx0 + (uint32_t)d0 * kHX, hy1 = hy0 + (uint32_t)d1 * kHY,
                        hz1 = hz0 + (uint32_t)d2 * kHZ;
         // cell c + (b0 d0, b1 d1, b2 d2), b = 1..7, exists iff every axis set in b has d != 0;
@@ -630,9 +571,6 @@ __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
     const uint32_t bx = blockIdx.x;
     const uint32_t nbA = (uint32_t)a.nbA, nbB = (uint32_t)a.nbB, nbC = (uint32_t)a.nbC;
     const uint32_t nA = (uint32_t)a.build_B * nbA, nB = (uint32_t)a.build_B * nbB;
-#ifdef CD_ABL_NO_BUILD
-    if (bx < nA + nB) return;
-#endif
     // Programmatic dependent launch (chained grid, StepArgs::pdl): build blocks depend on no
     // earlier launch still running -- the head/entry sets they write were last read two launches
     // ago, and this launch started only after every block of the previous one had triggered,
@@ -664,9 +602,6 @@ __global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
         if (!kChained)   // chained heads are epoch-tagged: nothing to clear
             for (int64_t i = tid; i < nw4; i += nth) zb[i] = make_uint4(0u, 0u, 0u, 0u);
         if (a.scan_B == 0) return;
-#ifdef CD_ABL_NO_SCAN
-        return;
-#endif
         const int s = (int)(b3 / nbC);
         const int64_t r = (int64_t)(b3 % nbC) * 256 + threadIdx.x;
         const bool stage = a.g.stage != 0;   // uniform over the launch

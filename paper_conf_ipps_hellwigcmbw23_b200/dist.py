@@ -90,11 +90,18 @@ FAR_KM = 1.0e9   # upper bound of the outermost shard (cd_options.shell_hi must 
 
 
 def shell_bounds(pop, S: int):
-    """S radial bands [b_s, b_{s+1}) with b_0 = 0, b_S = FAR_KM, balanced by the objects' mean
-    radius a (quantiles): each shard owns ~n/S objects."""
+    """At most S radial bands [b_s, b_{s+1}) with b_0 = 0, b_last = FAR_KM, balanced by the
+    objects' mean radius a (quantiles): each shard owns ~n/S objects.  The edges are strictly
+    increasing: quantiles that coincide (many objects with one a) merge their bands, as the
+    library's own band split does, so there may be fewer than S bands -- iterate over
+    len(bounds) - 1."""
     a = np.sort(np.asarray(pop["a"], dtype=np.float64))
-    inner = [float(a[min(len(a) - 1, (len(a) * s) // S)]) for s in range(1, S)]
-    return [0.0] + inner + [FAR_KM]
+    edges = [0.0]
+    for s in range(1, S):
+        q = float(a[min(len(a) - 1, (len(a) * s) // S)])
+        if q > edges[-1]:
+            edges.append(q)
+    return edges + [FAR_KM]
 
 
 def screen_shard(pop, t0, t1, dt, d, bounds, s, mode="grid", v_margin=7.8, **kw):

@@ -43,7 +43,7 @@ def test_exports_every_declared_symbol(cds):
 
 
 def test_version_status_options(cds):
-    assert cds.cd_abi_version() == 2
+    assert cds.cd_abi_version() == cds.ABI_VERSION
     assert cds.status_str(cds.CD_EINVAL) == "CD_EINVAL"
     assert cds.status_str(cds.CD_ENODEV) == "CD_ENODEV"
     o = cds.cd_options()
@@ -74,6 +74,17 @@ def test_no_cpu_fallback(cds):
     with pytest.raises(cds.CdError) as ei:
         cds.propagate(pop, [0.0])
     assert ei.value.status == cds.CD_ENODEV
+
+
+def test_option_validation_before_device(cds):
+    """Invalid options are CD_EINVAL on any machine (validated before a device is touched)."""
+    pop = {k: np.ones(4) * v for k, v in zip(cds.FIELDS, (7000.0, 0.001, 1, 1, 1, 1))}
+    for kw in (dict(kepler_points=5), dict(kepler_points=-4), dict(cell_factor=0.5),
+               dict(rank=2, n_ranks=2)):
+        with pytest.raises(cds.CdError) as ei:
+            cds.screen(pop, 0.0, 10.0, 1.0, 2.0, **kw)
+        assert ei.value.status == cds.CD_EINVAL, kw
+    assert cds.cd_release_caches(-1) == cds.CD_OK or _has_gpu()
 
 
 def test_product_never_imports_oracle():

@@ -159,3 +159,35 @@ def test_shell_bounds_and_members():
             assert np.array_equal(idx, want.astype(np.uint32))
     with pytest.raises(cds.CdError):
         cds.shell_members(pop, 7000.0, 7000.0, 1.0)
+
+
+def test_shell_bounds_merge_duplicate_quantiles():
+    """Many objects with one a (a shell): coinciding quantiles merge bands instead of producing an
+    empty band [b, b) (which cd_shell_members rejects); the bands still partition [0, inf)."""
+    import paper_conf_ipps_hellwigcmbw23_b200 as cds
+    from tools import popgen
+    pop = popgen.random_population(2000, 23, "catalog", 0)
+    pop["a"][:1400] = 7000.0
+    b = cdist.shell_bounds(pop, 8)
+    assert b[0] == 0.0 and b[-1] == cdist.FAR_KM
+    assert all(x < y for x, y in zip(b, b[1:]))
+    assert len(b) - 1 < 8
+    own = np.histogram(pop["a"], bins=b)[0]
+    assert own.sum() == 2000
+    for s in range(len(b) - 1):
+        cds.shell_members(pop, b[s], b[s + 1], 9.8)   # no CD_EINVAL
+
+
+def test_elements_validation():
+    """The binding checks the layout cdscreen.h assumes before any pointer reaches C."""
+    import paper_conf_ipps_hellwigcmbw23_b200 as cds
+    from tools import popgen
+    pop = popgen.random_population(100, 24, "catalog", 0)
+    bad = dict(pop, e=pop["e"][:50])
+    with pytest.raises(ValueError, match="different lengths"):
+        cds._Elements(bad)
+    bad = dict(pop, inc=np.stack([pop["inc"], pop["inc"]]))
+    with pytest.raises(ValueError, match="1-D"):
+        cds._Elements(bad)
+    E = cds._Elements(dict(pop, a=pop["a"].astype(np.float32)))   # host arrays are converted
+    assert E.n == 100 and E.keep[0].dtype == np.float64

@@ -63,3 +63,72 @@ def test_two_objects_crossing():
     assert abs(rows["grid"]["tca"] - rows["legacy"]["tca"]) < 1e-6
     assert abs(rows["grid"]["tca"] - rows["hybrid"]["tca"]) < 1e-3
     assert abs(rows["grid"]["pca"] - rows["hybrid"]["pca"]) < 1e-6
+
+
+def test_geo_at_small_cell_fits_21bit_keys():
+    """Cell keys pack 21 bits per axis (cdscreen.h CD_ERANGE): GEO objects at g_c = 0.1 km with
+    the paper's cell edge (L = g_c) sit ~421,640 cells from the origin -- beyond the 2^18 of a
+    19-bit key, inside 2^20 - 2.  Both grid structures, against brute force."""
+    rng = np.random.default_rng(11)
+    n = 400
+    # a GEO-belt cluster with close neighbours (small offsets in longitude and radius)
+    pop = {"a": 42164.0 + rng.uniform(-0.05, 0.05, n), "e": rng.uniform(0, 1e-5, n),
+           "inc": rng.uniform(0, 1e-4, n), "raan": rng.uniform(0, 2 * np.pi, n),
+           "argp": rng.uniform(0, 2 * np.pi, n), "nu0": rng.uniform(0, 2e-4, n)}
+    d, dt = 0.1, 1.0
+    gc = oracle.cell_size(d, dt, v_margin=0.0)
+    Ko = oracle.candidates_brute(pop, 0.0, 20.0, dt, gc)
+    assert len(Ko) > 0
+    for table in (1, 2):
+        Kg = cds.candidates(pop, 0.0, 20.0, dt, d, v_margin=0.0, cell_factor=1.0, grid_table=table)
+        parity.compare_candidates(pop, Kg, Ko, 0.0, dt, gc)
+
+
+def test_kepler_points_option():
+    """cd_options.kepler_points: a minimum Contour point count for every object -- the same
+    positions (1e-9) and candidate set; an unsupported count is CD_EINVAL."""
+    pop = popgen.random_population(3000, 12, "paper", 200)
+    times = np.array([0.0, 517.25, 86400.0])
+    xo = oracle.propagate(pop, times)
+    for kp in (8, 16):
+        xg = cds.propagate(pop, times, kepler_points=kp)
+        rel = np.linalg.norm(xg - xo, axis=2) / np.linalg.norm(xo, axis=2)
+        assert rel.max() < 1e-9, (kp, rel.max())
+    gc = oracle.cell_size(20.0, 1.0)
+    Ko = oracle.candidates_grid(pop, 0.0, 30.0, 1.0, gc)
+    Kg = cds.candidates(pop, 0.0, 30.0, 1.0, 20.0, kepler_points=12)
+    parity.compare_candidates(pop, Kg, Ko, 0.0, 1.0, gc)
+    with pytest.raises(cds.CdError) as ei:
+        cds.propagate(pop, times, kepler_points=5)
+    assert ei.value.status == cds.CD_EINVAL
+
+
+def test_device_inputs_validation_and_streams():
+    """CUDA-tensor inputs: fp64 / 1-D / one device are required (ValueError before C); inputs
+    written on a side stream are screened on that stream (the binding passes torch's current
+    stream), so the result equals the host-input result."""
+    import torch
+    pop = popgen.random_population(2000, 13)
+    host = cds.screen(pop, 0.0, 60.0, 1.0, 20.0)
+    bad = {k: torch.from_numpy(v).cuda() for k, v in pop.items()}
+    bad["a"] = bad["a"].float()
+    with pytest.raises(ValueError, match="float64"):
+        cds.screen(bad, 0.0, 60.0, 1.0, 20.0)
+    side = torch.cuda.Stream()
+    with torch.cuda.stream(side):
+        dev = {k: torch.empty(len(v), dtype=torch.float64, device="cuda") for k, v in pop.items()}
+        for k, v in pop.items():
+            dev[k].copy_(torch.from_numpy(v), non_blocking=True)
+        got = cds.screen(dev, 0.0, 60.0, 1.0, 20.0)
+    assert np.array_equal(got, host)
+
+
+def test_release_caches():
+    pop = popgen.random_population(2000, 14)
+    a = cds.screen(pop, 0.0, 60.0, 1.0, 20.0)
+    cds.release_caches()
+    cds.release_caches(0)
+    b = cds.screen(pop, 0.0, 60.0, 1.0, 20.0)
+    assert np.array_equal(a, b)
+    with pytest.raises(cds.CdError):
+        cds.release_caches(4096)
