@@ -72,9 +72,9 @@ def test_geo_at_small_cell_fits_21bit_keys():
     rng = np.random.default_rng(11)
     n = 400
     # a GEO-belt cluster with close neighbours (small offsets in longitude and radius)
-    pop = {"a": 42164.0 + rng.uniform(-0.05, 0.05, n), "e": rng.uniform(0, 1e-5, n),
-           "inc": rng.uniform(0, 1e-4, n), "raan": rng.uniform(0, 2 * np.pi, n),
-           "argp": rng.uniform(0, 2 * np.pi, n), "nu0": rng.uniform(0, 2e-4, n)}
+    pop = {"a": 42164.0 + rng.uniform(-0.05, 0.05, n), "e": rng.uniform(0, 1e-7, n),
+           "inc": rng.uniform(0, 1e-6, n), "raan": np.zeros(n),
+           "argp": np.zeros(n), "nu0": rng.uniform(0, 2e-4, n)}
     d, dt = 0.1, 1.0
     gc = oracle.cell_size(d, dt, v_margin=0.0)
     Ko = oracle.candidates_brute(pop, 0.0, 20.0, dt, gc)
