@@ -365,6 +365,12 @@ __device__ __forceinline__ void walk(const GridGeom& g, const Entry* __restrict_
 
 // Scan one object against the cells listed by (dx, dy, dz) offsets of its own cell: every bitmap
 // load is issued before any is resolved; set bits probe the table and walk the cell's list.
+// Measured alternatives on the hybrid's dense coarse grid (1M objects, g_c,h = 72.2 km; DESIGN.md
+// section 6): a flattened single loop (one entry or one slot probe per iteration, lanes kept
+// converged) ran 411 vs 324 us per step -- lockstep iterations wait for the slowest lane's
+// dependent load, while these nested loops let a warp's diverged lanes overlap their latencies;
+// an apogee/perigee gate in test_pair (the AP filter's rejections, 32 % of the candidates, not
+// queued) did not pay: 446 -> 451 us scan, 161 -> 165 us filter per step.
 __device__ __forceinline__ void probe_cell(const GridGeom& g, const Slot* __restrict__ slots,
                                            uint64_t mask, uint32_t tag, int cx, int cy, int cz,
                                            const Entry* __restrict__ E, uint32_t r, const double p[3],

@@ -33,9 +33,21 @@ GOLDEN = ROOT / "tests" / "golden"
 JOBS = {"cfg2_grid": (2, "grid"), "cfg2_hybrid": (2, "hybrid"), "cfg3_hybrid": (3, "hybrid")}
 
 
+def _sorted_by_ij(c):
+    if len(c) < 2:
+        return True
+    i, j = c["i"].astype(np.int64), c["j"].astype(np.int64)
+    di = np.diff(i)
+    return bool(np.all((di > 0) | ((di == 0) & (np.diff(j) >= 0))))
+
+
 def step_digests(cands, K):
-    """(count, digest) per step of a candidate array (any order)."""
-    order = np.lexsort((cands["j"], cands["i"], cands["step"]))
+    """(count, digest) per step of a candidate array (any order; an array already sorted by
+    (i, j) -- both sides' native order -- takes one stable sort by step)."""
+    if _sorted_by_ij(cands):
+        order = np.argsort(cands["step"], kind="stable")
+    else:
+        order = np.lexsort((cands["j"], cands["i"], cands["step"]))
     c = cands[order]
     bounds = np.searchsorted(c["step"], np.arange(K + 1))
     count = np.diff(bounds).astype(np.int64)
