@@ -370,7 +370,10 @@ __device__ __forceinline__ void walk(const GridGeom& g, const Entry* __restrict_
 // converged) ran 411 vs 324 us per step -- lockstep iterations wait for the slowest lane's
 // dependent load, while these nested loops let a warp's diverged lanes overlap their latencies;
 // an apogee/perigee gate in test_pair (the AP filter's rejections, 32 % of the candidates, not
-// queued) did not pay: 446 -> 451 us scan, 161 -> 165 us filter per step.
+// queued) did not pay: 446 -> 451 us scan, 161 -> 165 us filter per step; 16 lanes per object,
+// one half-shell cell each (more loads in flight, 16x the per-lane set-up), 432 vs 282 us; and
+// fewer blocks per SM for a spill-free open-map instance (CD_OPEN_MINB 5 / 4 / 3: 48 / 61 / 61
+// registers), 301 / 356 / 354 vs 282 us -- occupancy outweighs the spills.
 __device__ __forceinline__ void probe_cell(const GridGeom& g, const Slot* __restrict__ slots,
                                            uint64_t mask, uint32_t tag, int cx, int cy, int cz,
                                            const Entry* __restrict__ E, uint32_t r, const double p[3],
@@ -571,8 +574,11 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
 #ifndef CD_STEP_MINB
 #define CD_STEP_MINB 6
 #endif
+#ifndef CD_OPEN_MINB
+#define CD_OPEN_MINB 6
+#endif
 template <bool kChained, int kJ2>
-__global__ void __launch_bounds__(256, CD_STEP_MINB) k_step(StepArgs a)
+__global__ void __launch_bounds__(256, kChained ? CD_STEP_MINB : CD_OPEN_MINB) k_step(StepArgs a)
 {
     const uint32_t bx = blockIdx.x;
     const uint32_t nbA = (uint32_t)a.nbA, nbB = (uint32_t)a.nbB, nbC = (uint32_t)a.nbC;
