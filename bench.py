@@ -177,7 +177,11 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
+    # the distributed data plane (NCCL process group, per-slice all-gather merge, max-over-ranks
+    # timing) runs whenever there are several ranks, and also at one rank with --dist (torchrun
+    # --nproc-per-node 1), so a one-GPU box exercises the same code path
+    distributed = world > 1 or args.dist
+    if distributed:
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     else:
@@ -194,11 +198,16 @@ def run_ours(args):
     stream = torch.cuda.current_stream(dev)
 
     def barrier():
-        if world > 1:
+        if distributed:
             dist.barrier()
 
     # device scratch memory from PyTorch's caching allocator on the bench stream (cd_options.alloc)
     talloc = cds.TorchAllocator(dev.index, stream.cuda_stream) if args.torch_alloc else None
+
+    # the cell edge the first call settles on is passed to the next calls (cd_stats.cell_factor
+    # -> cd_options.cell_factor): later slices skip the density-probe round
+    cell = {"grid": None}
+    last_merged = {}
 
     def one_step(s, profile, host_inputs=False):
         q = (s * world + rank) % S
@@ -207,7 +216,7 @@ def run_ours(args):
         opt = cds.make_options(rank=q, n_ranks=S, device=dev.index, stream=stream.cuda_stream,
                                inputs_on_device=not host_inputs,
                                outputs_on_device=not host_inputs, profile_phases=profile,
-                               allocator=talloc)
+                               allocator=talloc, cell_factor=cell["grid"])
         import ctypes as C
         opt.stats = C.pointer(st)
         out = cds.cd_conjunctions()
@@ -218,12 +227,15 @@ def run_ours(args):
                 merged = nrec
             else:
                 recs = cdist.device_records_to_tensor(out, dev)
-                if world > 1:
+                if distributed:   # the slices of all ranks, merged and sorted on every rank
                     recs = cdist.merge_conjunctions(recs, stream=stream.cuda_stream)
+                    last_merged["recs"] = recs
                 merged = recs.shape[0]
                 nrec = int(out.count)
         finally:
             cds.cd_conjunctions_free(out)
+        if st.cell_factor > 0 and cell["grid"] is None:
+            cell["grid"] = float(st.cell_factor)
         return st.as_dict(), nrec, merged
 
     # the clock sampler starts before the warm-up so its NVML start-up does not land in the
@@ -261,7 +273,14 @@ def run_ours(args):
     clk.__exit__(None, None, None)
     launches = cds.cd_kernel_launches() - launches0
     tot_ms = float(np.sum(times))
-    if world > 1:
+    merge_info = None
+    if distributed:
+        recs = last_merged.get("recs")
+        dups = cdist.count_duplicates(recs) if recs is not None else 0
+        merge_info = {"backend": dist.get_backend(), "ranks": world,
+                      "records_last_step": int(recs.shape[0]) if recs is not None else 0,
+                      "duplicates_last_step": int(dups)}
+    if distributed:
         t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         tot_ms = float(t.item())
@@ -269,7 +288,7 @@ def run_ours(args):
         dist.all_reduce(c)
         nconj = int(c.item())
     units = float(n) * sum(st["steps"] for st in stats) * 1.0
-    if world > 1:
+    if distributed:
         u = torch.tensor([units], dtype=torch.float64, device=dev)
         dist.all_reduce(u)
         units = float(u.item())
@@ -285,7 +304,8 @@ def run_ours(args):
             E = cds._Elements(dpop)
             st = cds.cd_stats()
             opt = cds.make_options(rank=q, n_ranks=S, device=dev.index, stream=stream.cuda_stream,
-                                   inputs_on_device=True, outputs_on_device=True, allocator=talloc)
+                                   inputs_on_device=True, outputs_on_device=True, allocator=talloc,
+                                   cell_factor=cell.get("hybrid"))
             import ctypes as C
             opt.stats = C.pointer(st)
             out = cds.cd_conjunctions()
@@ -298,16 +318,18 @@ def run_ours(args):
             cds._check(cds.cd_screen_ex(E.s, E.n, cfg.t0, cfg.t1, cfg.dt_hybrid, cfg.d, cds.CD_HYBRID,
                                         opt, out))
             recs = cdist.device_records_to_tensor(out, dev)
-            if world > 1:
+            if distributed:
                 recs = cdist.merge_conjunctions(recs, stream=stream.cuda_stream)
             cds.cd_conjunctions_free(out)
+            if st.cell_factor > 0 and cell.get("hybrid") is None:
+                cell["hybrid"] = float(st.cell_factor)
             e1.record(stream)
             torch.cuda.synchronize()
             if s >= args.warmup:
                 hms.append(e0.elapsed_time(e1))
                 hst.append(st.as_dict())
         htot = float(np.sum(hms))
-        if world > 1:
+        if distributed:
             t = torch.tensor([htot], dtype=torch.float64, device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             htot = float(t.item())
@@ -321,7 +343,10 @@ def run_ours(args):
                           ("hybrid_ap_rejected", "hybrid_coplanar", "hybrid_path_rejected",
                            "hybrid_time_rejected", "refined")}}
 
-    # end to end through the public API with HOST buffers (pinned inputs, results to host)
+    # end to end through the public API with HOST buffers: pinned host inputs (H2D inside the
+    # call), results back in host memory.  One rank: cd_screen with host results.  Distributed:
+    # each rank's slice stays on the device for the NCCL merge (all-gather + device sort), and
+    # the merged, sorted result is copied to the host (D2H inside the timed region).
     e2e_ms = []
     pin = {k: torch.from_numpy(v).pin_memory() for k, v in pop.items()}
     pin_np = {k: v.numpy() for k, v in pin.items()}
@@ -334,15 +359,28 @@ def run_ours(args):
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         q = (s * world + rank) % S
-        recs = cds.screen(pin_np, cfg.t0, cfg.t1, dt, cfg.d, mode=args.variant, rank=q, n_ranks=S,
-                          device=dev.index, stream=stream.cuda_stream, allocator=talloc)
+        if distributed:
+            E = cds._Elements(pin_np)
+            opt = cds.make_options(rank=q, n_ranks=S, device=dev.index, stream=stream.cuda_stream,
+                                   outputs_on_device=True, allocator=talloc, cell_factor=cell["grid"])
+            out = cds.cd_conjunctions()
+            cds._check(cds.cd_screen_ex(E.s, E.n, cfg.t0, cfg.t1, dt, cfg.d, mode, opt, out))
+            recs = cdist.merge_conjunctions(cdist.device_records_to_tensor(out, dev),
+                                            stream=stream.cuda_stream)
+            cds.cd_conjunctions_free(out)
+            host = cdist.records_to_numpy(recs)
+            d2h += host.nbytes
+        else:
+            recs = cds.screen(pin_np, cfg.t0, cfg.t1, dt, cfg.d, mode=args.variant, rank=q, n_ranks=S,
+                              device=dev.index, stream=stream.cuda_stream, allocator=talloc,
+                              cell_factor=cell["grid"])
+            d2h += recs.nbytes
         e1.record(stream)
         torch.cuda.synchronize()
         e2e_ms.append(e0.elapsed_time(e1))
-        d2h += recs.nbytes
     ne2e = len(e2e_ms)
     e2e_tot = float(np.sum(e2e_ms))
-    if world > 1:
+    if distributed:
         t = torch.tensor([e2e_tot], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_tot = float(t.item())
@@ -352,7 +390,7 @@ def run_ours(args):
            "steps": ne2e}
 
     if rank != 0:
-        if world > 1:
+        if distributed:
             dist.destroy_process_group()
         return 0
 
@@ -404,9 +442,9 @@ def run_ours(args):
             "step_ms": {"min": float(np.min(times)), "median": float(np.median(times)),
                         "max": float(np.max(times))},
             "clocks": clk.summary(), "e2e": e2e, "gpu_launches": launches,
-            "roofline": roof, "cpu_baseline": cpu, "hybrid": hyb}
+            "roofline": roof, "cpu_baseline": cpu, "hybrid": hyb, "merge": merge_info}
     print(json.dumps(line), flush=True)
-    if world > 1:
+    if distributed:
         dist.destroy_process_group()
     return 0
 
@@ -438,6 +476,8 @@ def main():
     ap.add_argument("--cpu-steps", type=int, default=128)
     ap.add_argument("--ref-steps", type=int, default=None)
     ap.add_argument("--e2e-steps", type=int, default=None)
+    ap.add_argument("--dist", action="store_true",
+                    help="NCCL process group + merge even at one rank (torchrun --nproc-per-node 1)")
     ap.add_argument("--no-torch-alloc", dest="torch_alloc", action="store_false",
                     help="library's own stream-ordered pool instead of PyTorch's caching allocator")
     args = ap.parse_args()

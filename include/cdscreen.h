@@ -52,7 +52,8 @@
 extern "C" {
 #endif
 
-#define CD_ABI_VERSION 3   /* 2: cd_options.propagator; 3: kepler_points honoured, cd_release_caches */
+#define CD_ABI_VERSION 3   /* 2: cd_options.propagator; 3: kepler_points honoured, cd_release_caches,
+                              cd_stats.cell_factor / grid_table */
 
 typedef enum {
     CD_OK = 0,
@@ -148,6 +149,11 @@ typedef struct {
     double ms_clear, ms_propagate, ms_insert, ms_scan, ms_refine, ms_finalize, ms_precompute;
     uint64_t launches_clear, launches_propagate, launches_insert, launches_scan, launches_refine;
     uint64_t step_launches;    /* all launches of the fused step kernel (timed or not)         */
+    double cell_factor;        /* the cell edge L / g_c the call settled on (auto: chosen from the
+                                  measured candidate density).  Passing it back as
+                                  cd_options.cell_factor to the next call over the same population
+                                  (e.g. the next time slice) skips that call's density-probe round */
+    int grid_table;            /* the grid structure the call used: 1 open addressing, 2 chained  */
 } cd_stats;
 
 typedef struct {

@@ -75,7 +75,7 @@ class cd_stats(C.Structure):
                 ("ms_precompute", C.c_double), ("launches_clear", C.c_uint64),
                 ("launches_propagate", C.c_uint64), ("launches_insert", C.c_uint64),
                 ("launches_scan", C.c_uint64), ("launches_refine", C.c_uint64),
-                ("step_launches", C.c_uint64)]
+                ("step_launches", C.c_uint64), ("cell_factor", C.c_double), ("grid_table", C.c_int)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -1115,6 +1115,8 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         }
     }
     R.n_conj = (size_t)conj_before;
+    stats.cell_factor = L / gc;
+    stats.grid_table = chained ? 2 : 1;
     stats.hybrid_ap_rejected = hyb_before[0];
     stats.hybrid_coplanar = hyb_before[1];
     stats.hybrid_path_rejected = hyb_before[2];

@@ -65,6 +65,17 @@ def merge_conjunctions(local, group=None, stream=None):
     return allrec
 
 
+def count_duplicates(recs):
+    """Rows of a merged, sorted record tensor (m, 32) whose (i, j, step) equals the previous
+    row's.  Under the owner rule every minimum belongs to exactly one slice, so a correct merge
+    has none (the north star's dedupe step is this check)."""
+    import torch
+    if recs is None or recs.shape[0] < 2:
+        return 0
+    key = recs[:, :12].contiguous().view(torch.int32).view(-1, 3)
+    return int((key[1:] == key[:-1]).all(dim=1).sum().item())
+
+
 def device_records_to_tensor(out, device):
     """Copy a library-owned device result (cd_conjunctions with outputs_on_device) into a torch
     uint8 tensor (m, 32) on `device`."""

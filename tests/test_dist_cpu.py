@@ -50,6 +50,19 @@ def _worker(rank, world, port, t1, d, ret):
         dist.destroy_process_group()
 
 
+def test_count_duplicates():
+    """The merge's dedupe check (dist.count_duplicates) on sorted 32-byte records."""
+    recs = np.zeros(5, dtype=[("i", "<u4"), ("j", "<u4"), ("step", "<u4"), ("flags", "<u4"),
+                              ("tca", "<f8"), ("pca", "<f8")])
+    recs["i"] = [1, 1, 1, 2, 2]
+    recs["j"] = [3, 3, 4, 5, 5]
+    recs["step"] = [7, 8, 8, 9, 9]
+    t = torch.from_numpy(np.frombuffer(recs.tobytes(), dtype=np.uint8).reshape(-1, 32).copy())
+    assert cdist.count_duplicates(t) == 1
+    assert cdist.count_duplicates(t[:4]) == 0
+    assert cdist.count_duplicates(t[:1]) == 0
+
+
 @pytest.mark.parametrize("world", [2, 3])
 def test_slices_gather_equals_whole_window(orc, world):
     t1, d = 80.0, 10.0
