@@ -211,6 +211,12 @@ typedef struct {
                                  with n/S plus the halo; the union is exactly the unsharded
                                  result.  0 or 1 = off (default; at 8M objects on one B200 the
                                  bands were measured 1-14 % slower), <= 64                        */
+    int resort_steps;         /* spatial slot order: every R sampling steps the objects are
+                                 renumbered in Morton order of their current position, so the
+                                 grid accesses of neighbouring threads are neighbours in memory
+                                 (results do not depend on it).  0 = auto (default: every
+                                 max(16, 64 s / dt) steps for >= 4M objects in CD_GRID, else
+                                 off), < 0 = off, R > 0 = every R steps                         */
 } cd_options;
 
 /* Fill *opt with the defaults above. */

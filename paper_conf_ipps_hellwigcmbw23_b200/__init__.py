@@ -95,7 +95,7 @@ class cd_options(C.Structure):
                 ("stats", C.POINTER(cd_stats)), ("propagator", C.c_int),
                 ("shell_lo", C.c_double), ("shell_hi", C.c_double),
                 ("alloc", ALLOC_FN), ("free", FREE_FN), ("alloc_ctx", C.c_void_p),
-                ("shards", C.c_int)]
+                ("shards", C.c_int), ("resort_steps", C.c_int)]
 
 
 class cd_plan_info(C.Structure):
@@ -314,7 +314,7 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
                  cell_factor=None, batch_object_steps=None, round_steps=None,
                  outputs_on_device=False, inputs_on_device=False, profile_phases=False,
                  l2_persist=None, grid_table=None, propagator=None, shell=None, allocator=None,
-                 shards=None, kepler_points=None):
+                 shards=None, kepler_points=None, resort_steps=None):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -357,6 +357,8 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
         o.shards = int(shards)
     if kepler_points is not None:
         o.kepler_points = int(kepler_points)
+    if resort_steps is not None:
+        o.resort_steps = int(resort_steps)
     return o
 
 

@@ -140,6 +140,20 @@ cudaError_t finalize_conj(const cdk::Conj* in, size_t count, const uint32_t* per
                           cudaStream_t st, LaunchCount& lc);
 cudaError_t finalize_cand(const cdk::Cand* in, size_t count, const uint32_t* perm, cdk::Cand* out,
                           cudaStream_t st, LaunchCount& lc);
+// spatial slot order (cd_sort.cu): scratch of one re-sort, allocated once per call
+struct SpaceSort {
+    unsigned long long *key, *key2;
+    uint32_t *val, *val2;
+    void* tmp;
+    size_t tmp_bytes;
+};
+cudaError_t space_sort_temp_bytes(int64_t n, size_t* bytes);
+// renumber the n slots in Morton order (within class) of the positions in E (one built step,
+// slot-indexed in the old order); gather the old hot build records / classes / slot -> internal
+// id map (sold: nullptr = identity) into the new order
+cudaError_t space_resort(const SpaceSort& S, const cdk::Entry* E, const double* Hold, const uint8_t* cold,
+                         const uint32_t* sold, int64_t n, int ncol, int j2, double* Hnew,
+                         uint8_t* cnew, uint32_t* snew, cudaStream_t st, LaunchCount& lc);
 // stable sort of (key, value) pairs with CUB, used by classify
 cudaError_t sort_pairs_u32(const uint32_t* kin, uint32_t* kout, const uint32_t* vin, uint32_t* vout,
                            size_t count, int end_bit, cudaStream_t st, LaunchCount& lc);

@@ -331,9 +331,10 @@ __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_
         const double rb = fma(ej.x, ej.x, fma(ej.y, ej.y, ej.z * ej.z));
         const double rm = fmin(ra, rb);
         if (!(rm >= g.band_lo2 && rm < g.band_hi2)) return;
+        const uint32_t a = g.sig ? g.sig[r] : r, b = g.sig ? g.sig[j] : j;   // slots -> internal ids
         Cand cd;
-        cd.i = r < j ? r : j;
-        cd.j = r < j ? j : r;
+        cd.i = a < b ? a : b;
+        cd.j = a < b ? b : a;
         cd.step = step;
         if (g.stage) {
             const unsigned w = threadIdx.x >> 5;

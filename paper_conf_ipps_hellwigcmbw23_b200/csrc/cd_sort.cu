@@ -121,6 +121,84 @@ static cudaError_t finalize_impl(const Rec* in, size_t n, const uint32_t* perm, 
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------------------------------
+// Spatial slot order (DESIGN.md section 5 "Spatial order"): every R steps the objects are
+// renumbered in Morton order of their current position (within their eccentricity class), so a
+// warp's objects -- and the grid heads, cells and list entries they touch -- are neighbours in
+// space and memory.  The hot build records, the class bytes and the slot -> internal id map are
+// gathered into the new order.
+// ---------------------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t spread3(uint32_t v)   // 16 bits -> every third of 48
+{
+    uint64_t x = v & 0xffffu;
+    x = (x | (x << 32)) & 0x1f00000000ffffull;
+    x = (x | (x << 16)) & 0x1f0000ff0000ffull;
+    x = (x | (x << 8)) & 0x100f00f00f00f00full;
+    x = (x | (x << 4)) & 0x10c30c30c30c30c3ull;
+    x = (x | (x << 2)) & 0x1249249249249249ull;
+    return x;
+}
+
+__device__ __forceinline__ uint32_t quant16(double x)   // [-65536, 65536) km in 2 km steps
+{
+    const double q = floor((x + 65536.0) * 0.5);
+    return q < 0.0 ? 0u : q > 65535.0 ? 65535u : (uint32_t)q;
+}
+
+__global__ void k_space_keys(const Entry* __restrict__ E, const uint8_t* __restrict__ cls, int64_t n,
+                             unsigned long long* __restrict__ key, uint32_t* __restrict__ val)
+{
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (t >= n) return;
+    const Entry e = E[t];
+    const uint64_t m = spread3(quant16(e.x)) | (spread3(quant16(e.y)) << 1) | (spread3(quant16(e.z)) << 2);
+    key[t] = ((unsigned long long)cls[t] << 48) | m;   // class first (class-0 slots stay [0, n0))
+    val[t] = (uint32_t)t;
+}
+
+// new slot u takes old slot t = perm[u]: its build-record columns (class 0: the 9 lean columns
+// plus the J2 rates; other classes: all), class byte and internal id
+__global__ void k_resort_gather(const double* __restrict__ Hold, const uint8_t* __restrict__ cold,
+                                const uint32_t* __restrict__ sold, const uint32_t* __restrict__ perm,
+                                int64_t n, int ncol, int j2, double* __restrict__ Hnew,
+                                uint8_t* __restrict__ cnew, uint32_t* __restrict__ snew)
+{
+    const int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (u >= n) return;
+    const uint32_t t = perm[u];
+    const uint8_t c = cold[t];
+    cnew[u] = c;
+    snew[u] = sold ? sold[t] : t;
+    const int lean = kBQz + 1;
+    for (int k = 0; k < (c == 0 ? lean : ncol); ++k) Hnew[k * n + u] = Hold[k * n + t];
+    if (c == 0 && j2)
+        for (int k = kDOm; k < ncol; ++k) Hnew[k * n + u] = Hold[k * n + t];
+}
+
+cudaError_t space_sort_temp_bytes(int64_t n, size_t* bytes)
+{
+    *bytes = 0;
+    return cub::DeviceRadixSort::SortPairs(nullptr, *bytes, (const unsigned long long*)nullptr,
+                                           (unsigned long long*)nullptr, (const uint32_t*)nullptr,
+                                           (uint32_t*)nullptr, n, 0, 51);
+}
+
+cudaError_t space_resort(const SpaceSort& S, const Entry* E, const double* Hold, const uint8_t* cold,
+                         const uint32_t* sold, int64_t n, int ncol, int j2, double* Hnew,
+                         uint8_t* cnew, uint32_t* snew, cudaStream_t st, LaunchCount& lc)
+{
+    const unsigned blocks = (unsigned)((n + 255) / 256);
+    k_space_keys<<<blocks, 256, 0, st>>>(E, cold, n, S.key, S.val);
+    lc.bump();
+    CD_TRY(cudaGetLastError());
+    size_t tb = S.tmp_bytes;
+    CD_TRY(cub::DeviceRadixSort::SortPairs(S.tmp, tb, S.key, S.key2, S.val, S.val2, n, 0, 51, st));
+    lc.bump(8);
+    k_resort_gather<<<blocks, 256, 0, st>>>(Hold, cold, sold, S.val2, n, ncol, j2, Hnew, cnew, snew);
+    lc.bump();
+    return cudaGetLastError();
+}
+
 cudaError_t finalize_conj(const Conj* in, size_t count, const uint32_t* perm, Conj* out,
                           cudaStream_t st, LaunchCount& lc)
 {

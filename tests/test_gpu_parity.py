@@ -279,3 +279,27 @@ def test_config5_8m_sampled_steps():
     # rows on one side only (a minimum just outside [t0, t1] taken for one) would hide here as
     # window-edge exclusions: the 2-s window has thousands of encounters straddling its ends
     assert parity.compare_conjunctions(pop, Cg, Co, t0, t1, dt, d, gc)["one_sided"] == 0
+
+
+@pytest.mark.parametrize("mode,dt,R", [("grid", 1.0, 1), ("grid", 1.0, 7), ("hybrid", 9.0, 2),
+                                       ("grid", 1.0, 3)])
+def test_spatial_resort_is_invisible(mode, dt, R):
+    """cd_options.resort_steps: renumbering the slots in Morton order every R steps (pipeline
+    double-buffered: a launch builds in the new order while it scans in the old) changes nothing
+    -- candidates and conjunctions identical to the unsorted screen and to the oracle."""
+    pop = _mix(20000, 31, "paper", 3000)
+    d = 8.0
+    t0, t1 = 200.0, 200.0 + 90 * dt
+    gc = oracle.cell_size(d, dt)
+    kw = dict(batch_object_steps=40000) if R == 3 else {}   # B = 2 steps per batch
+    K0 = cds.candidates(pop, t0, t1, dt, d, resort_steps=-1)
+    K1 = cds.candidates(pop, t0, t1, dt, d, resort_steps=R, **kw)
+    assert np.array_equal(K0, K1)
+    C0 = cds.screen(pop, t0, t1, dt, d, mode=mode, resort_steps=-1)
+    C1 = cds.screen(pop, t0, t1, dt, d, mode=mode, resort_steps=R, **kw)
+    assert np.array_equal(C0, C1)
+    if mode == "grid":
+        Ko = oracle.candidates_grid(pop, t0, t1, dt, gc)
+        parity.compare_candidates(pop, K1, Ko, t0, dt, gc)
+        Co = oracle.conjunctions(pop, t0, t1, dt, d, gc, Ko)
+        parity.compare_conjunctions(pop, C1, Co, t0, t1, dt, d, gc)

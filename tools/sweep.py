@@ -17,6 +17,8 @@ def main():
     ap.add_argument("--batch", default="0")
     ap.add_argument("--persist", default="0")
     ap.add_argument("--table", default="0")
+    ap.add_argument("--resort", default="0", help="cd_options.resort_steps values (0 auto, -1 off)")
+    ap.add_argument("--t0", type=float, default=3600.0)
     args = ap.parse_args()
     import torch
     import paper_conf_ipps_hellwigcmbw23_b200 as cds
@@ -24,14 +26,15 @@ def main():
     pop, cfg, _ = popgen.make_config(args.config, n=args.n)
     dt = cfg.dt_grid if args.variant == "grid" else cfg.dt_hybrid
     dpop = {k: torch.from_numpy(v).cuda() for k, v in pop.items()}
-    t0 = 3600.0
+    t0 = args.t0
     t1 = t0 + (args.steps - 1) * dt
     ref = None
-    for pers in [int(x) for x in args.persist.split(",")]:
-     for tbl in [int(x) for x in args.table.split(",")]:
-      for b in [int(x) for x in args.batch.split(",")]:
-        for cf in [float(x) for x in args.cell.split(",")]:
-            kw = dict(cell_factor=cf, profile_phases=True, l2_persist=pers, grid_table=tbl)
+    import itertools
+    ints = lambda x: [int(v) for v in x.split(",")]
+    for rs, pers, tbl, b, cf in itertools.product(ints(args.resort), ints(args.persist), ints(args.table),
+                                                  ints(args.batch), [float(v) for v in args.cell.split(",")]):
+            kw = dict(cell_factor=cf, profile_phases=True, l2_persist=pers, grid_table=tbl,
+                      resort_steps=rs)
             if b:
                 kw["batch_object_steps"] = b
             cds.screen(dpop, t0, t0 + 20 * dt, dt, cfg.d, mode=args.variant, **kw)  # warm
@@ -40,7 +43,8 @@ def main():
                 ref = res
             same = bool(len(res) == len(ref) and (res[["i", "j", "step"]] == ref[["i", "j", "step"]]).all())
             k = st["steps"]
-            out = {"cell": cf, "table": tbl, "batch": b, "persist": pers, "ms_per_step_total": st["ms_total"] / k,
+            out = {"resort": rs, "cell": cf, "table": tbl, "batch": b, "persist": pers,
+                   "ms_per_step_total": st["ms_total"] / k,
                    "us_clear": 1e3 * st["ms_clear"] / k, "us_prop": 1e3 * st["ms_propagate"] / k,
                    "us_insert": 1e3 * st["ms_insert"] / k, "us_scan": 1e3 * st["ms_scan"] / k,
                    "us_refine": 1e3 * st["ms_refine"] / k, "cand": st["candidates"],
