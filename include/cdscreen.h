@@ -153,7 +153,8 @@ typedef struct {
                                   measured candidate density).  Passing it back as
                                   cd_options.cell_factor to the next call over the same population
                                   (e.g. the next time slice) skips that call's density-probe round */
-    int grid_table;            /* the grid structure the call used: 1 open addressing, 2 chained  */
+    int grid_table;            /* the grid structure the call used: 1 open addressing, 2 chained,
+                                  3 CSR (sort + segment)                                          */
 } cd_stats;
 
 typedef struct {
@@ -181,7 +182,11 @@ typedef struct {
     int grid_table;           /* per-step grid structure: 1 = the paper's open-addressing hash
                                  map (64-bit keys, linear probing, CAS, per-cell lists);
                                  2 = chained spatial hash (lists per hashed bucket, one atomic
-                                 exchange per object); 0 = default (2).  Results are identical. */
+                                 exchange per object); 3 = sort + segment (the open-addressing
+                                 slots count each cell's objects, a counting sort by cell makes
+                                 each cell one contiguous segment); 0 = default (per geometry:
+                                 2 in ball mode, 1 in half-shell mode).  Results are identical;
+                                 other values CD_EINVAL.                                         */
     cd_stats* stats;          /* optional output                                              */
     int propagator;           /* cd_propagator; default CD_PROP_KEPLER                        */
     double shell_lo, shell_hi;/* radial shard [km] (object-space sharding for

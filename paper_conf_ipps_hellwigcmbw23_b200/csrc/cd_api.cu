@@ -451,6 +451,7 @@ cd_status validate_scalars(size_t n, double t0, double t1, double dt, double d, 
     if (o.propagator != CD_PROP_KEPLER && o.propagator != CD_PROP_J2)
         return fail(CD_EINVAL, "unknown propagator %d", o.propagator);
     if (o.shards < 0 || o.shards > 64) return fail(CD_EINVAL, "need 0 <= shards <= 64");
+    if (o.grid_table < 0 || o.grid_table > 3) return fail(CD_EINVAL, "grid_table %d: need 0..3", o.grid_table);
     if (kepler_class_of_points(o.kepler_points) < 0)
         return fail(CD_EINVAL, "kepler_points = %d: need 0 (per e) or 4, 6, 8, 12, 16", o.kepler_points);
     if ((o.alloc == nullptr) != (o.free == nullptr))
@@ -760,8 +761,11 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     // spatial hash (bucket heads only); 0 = per geometry: chained in ball mode (L >= 2 g_c, where
     // it is measured faster), open addressing in half-shell mode (L < 2 g_c, where chaining would
     // walk all 26 neighbour buckets from both sides).  Both are allocated under 0, so the mode
-    // can follow the cell edge chosen after the first round.
-    const bool can_chain = o.grid_table != 1, can_open = o.grid_table != 2;
+    // can follow the cell edge chosen after the first round.  3 = CSR grid (sort + segment: the
+    // open-addressing slots count each cell's objects, a counting sort makes each cell's entries
+    // one contiguous segment).
+    const bool csr = o.grid_table == 3;
+    const bool can_chain = o.grid_table != 1 && !csr, can_open = o.grid_table != 2;
 #ifndef CD_CHAIN_FACTOR
 #define CD_CHAIN_FACTOR 8
 #endif
@@ -790,6 +794,16 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     // while launch i may still scan batch b (and build b + 1)
     Entry* entbuf[3];
     for (int h = 0; h < 3; ++h) entbuf[h] = reinterpret_cast<Entry*>(arena.p + tab_bytes + h * ent_bytes);
+    // CSR grid: per-object (slot, rank) entries of the batch being built, segment starts per slot
+    // (two sets, like the slots), per-step object totals; the segments go to entbuf
+    DBuf<Entry> csr_tmp(st);
+    DBuf<uint32_t> csr_start(st);
+    DBuf<unsigned long long> csr_total(st);
+    if (csr) {
+        CU(csr_tmp.alloc((size_t)Bmax * n));
+        CU(csr_start.alloc(2 * (size_t)Bmax * M));
+        CU(csr_total.alloc((size_t)Bmax));
+    }
     static const bool no_pdl = getenv("CD_NO_PDL") != nullptr;   // A/B switch for experiments
     auto tab_of = [&](uint64_t b) {
         return GridTab{slotset[b % 2], bitset[b % 3],
@@ -890,7 +904,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     const int64_t resort_auto = (n >= 4000000 && mode == CD_GRID)
                                     ? std::max<int64_t>(16, (int64_t)std::llround(64.0 / dt)) : 0;
     const int64_t resort_R = rs_opt < 0 ? 0 : rs_opt > 0 ? rs_opt : resort_auto;
-    const bool spatial = resort_R > 0 && n >= 4096;
+    const bool spatial = resort_R > 0 && n >= 4096 && !csr;   // (CSR segments are cell-ordered)
     const int ncolH = S.j2 ? kNCol : kDOm;
     DBuf<double> Hrec[2] = {DBuf<double>(st), DBuf<double>(st)};
     DBuf<uint8_t> Hcls[2] = {DBuf<uint8_t>(st), DBuf<uint8_t>(st)};
@@ -987,7 +1001,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                 sa.build_k0 = kr + i * Bmax;
                 sa.build_B = std::min<int64_t>(Bmax, kr + Rk - sa.build_k0);
                 sa.build_tab = tab_of(bb);
-                sa.build_ents = entbuf[bb % 3];
+                sa.build_ents = csr ? csr_tmp.p : entbuf[bb % 3];
                 sa.build_tag = tag_of(bb);
                 batch_ver[bb % 3] = order_ver;
                 since_resort += sa.build_B;
@@ -999,7 +1013,9 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                 sa.scan_ents = entbuf[(bb - 1) % 3];
                 sa.scan_tag = tag_of(bb - 1);
                 sa.g.sig = sig_of(batch_ver[(bb - 1) % 3]);
+                if (csr) sa.scan_start = csr_start.p + ((bb - 1) % 2) * (size_t)Bmax * M;
             }
+            sa.csr = csr ? 1 : 0;
             sa.zero_bits = bitset[(bb + 1) % 3];   // batch bb - 2's bitmaps, next built by bb + 1
             sa.zero_bits_words = bwords;
             sa.zero_depth = chained ? 0 : Bmax;   // chained heads are epoch-tagged
@@ -1007,6 +1023,10 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             sa.pdl = chained && !no_pdl ? 1 : 0;
             if (i == 0) C.pt.span_start(kPhScan);
             CU(launch_step(sa, &win, st, C.lc));
+            if (csr && i < J)   // segments of the batch just built, for the next launch's scan
+                CU(launch_csr_segments(slotset[bb % 2], csr_start.p + (bb % 2) * (size_t)Bmax * M, M,
+                                       csr_tmp.p, entbuf[bb % 3], n, (int)sa.build_B, tag_of(bb),
+                                       csr_total.p, st, C.lc));
         }
         C.pt.span_stop((uint64_t)J + 1);
         batch_no += (uint64_t)J;
@@ -1178,7 +1198,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     }
     R.n_conj = (size_t)conj_before;
     stats.cell_factor = L / gc;
-    stats.grid_table = chained ? 2 : 1;
+    stats.grid_table = csr ? 3 : chained ? 2 : 1;
     stats.hybrid_ap_rejected = hyb_before[0];
     stats.hybrid_coplanar = hyb_before[1];
     stats.hybrid_path_rejected = hyb_before[2];

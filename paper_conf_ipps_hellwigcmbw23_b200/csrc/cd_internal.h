@@ -121,7 +121,14 @@ struct StepArgs {
     int64_t nCblocks;            // role-C blocks in the launch
     int chained;                 // 1: chained spatial hash (heads in the bitmap arrays)
     int pdl;                     // 1: programmatic dependent launch (chained grid only)
+    int csr;                     // 1: CSR grid (counting sort by cell): build_ents = per-object
+                                 // (slot, rank) entries, scan_ents = the scanned batch's segments
+    const uint32_t* scan_start;  // CSR: segment start per slot of the scanned batch
 };
+// CSR grid: segments of a built batch (B steps): k_csr_alloc + k_csr_scatter (cd_kernels.cu)
+cudaError_t launch_csr_segments(const cdk::Slot* slots, uint32_t* start, uint64_t M,
+                                const cdk::Entry* tmp, cdk::Entry* csr, int64_t n, int B, uint32_t tag,
+                                unsigned long long* total, cudaStream_t st, LaunchCount& lc);
 cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCount& lc);
 
 // ---- refinement (a7) -------------------------------------------------------------------

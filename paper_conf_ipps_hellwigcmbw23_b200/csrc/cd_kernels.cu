@@ -251,7 +251,39 @@ cudaError_t launch_conj_to_global(const Conj* in, size_t n, const uint32_t* perm
 // (Eq. 2) and its occupancy bitmap; the entry {x, y, z, next} (Fig. 6) is
 // written once, coalesced.  kClass0: objects [0, n0) (e <= 0.01: lean N = 4 Contour path).
 // ---------------------------------------------------------------------------------------
-template <bool kClass0, bool kChained, int kJ2>
+// Grid structures (cd_options.grid_table): kOpen = the paper's open-addressing map with per-cell
+// lists, kChained = chained spatial hash, kCsr = open-addressing map of per-cell counts plus a
+// counting sort of the entries by cell (sort + segment: each cell's objects contiguous).
+enum GridKind : int { kOpen = 0, kChained = 1, kCsr = 2 };
+
+// CSR grid insert: claim the cell's slot (128-bit CAS from a stale slot to {key, tag | 1}) or
+// count the object into it (64-bit atomicAdd on the head word; count in the low 32 bits).
+// Returns the slot; *rank = the object's position among its cell's objects.
+__device__ __forceinline__ uint32_t grid_count(Slot* slots, uint64_t mask, unsigned long long key,
+                                               uint32_t tag, uint32_t* rank)
+{
+    const unsigned long long th = (unsigned long long)tag << 32;
+    uint64_t h = fmix64(key) & mask;
+    while (true) {
+        unsigned long long w0, w1;
+        asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(w0), "=l"(w1) : "l"(slots + h));
+        while (true) {
+            const bool stale = (uint32_t)(w1 >> 32) != tag;
+            if (!stale && w0 != key) break;   // another cell of this pass: next slot (Eq. 2)
+            if (!stale) {
+                *rank = (uint32_t)atomicAdd(&slots[h].head, 1ull);
+                return (uint32_t)h;
+            }
+            if (cas128(slots + h, w0, w1, key, th | 1ull)) {
+                *rank = 0;
+                return (uint32_t)h;
+            }
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+template <bool kClass0, int kGrid, int kJ2>
 __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, const GridTab& tab,
                                          Entry* __restrict__ ents, uint64_t mask, int64_t k0, int s,
                                          int64_t r, double t0, double dt, uint32_t tag, Ctrl* ctrl)
@@ -261,7 +293,12 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
     state<false, kClass0 ? 0 : -1, kJ2>(O, r, t, p, v);
     int c[3];
     uint32_t next = kNil, ctag = 0;
-    if (kChained && cell_of(g, p, c)) {
+    if (kGrid == kCsr && cell_of(g, p, c)) {
+        // counting insert; the entry (slot, rank) is scattered to its cell's segment later
+        const uint32_t hb = bit_hash(c[0], c[1], c[2]) & tab.bmask;
+        atomicOr(tab.bits + (size_t)s * tab.bwords + (hb >> 5), 1u << (hb & 31));
+        next = grid_count(tab.slots + (size_t)s * (mask + 1), mask, pack_key(c[0], c[1], c[2]), tag, &ctag);
+    } else if (kGrid == kChained && cell_of(g, p, c)) {
         ctag = cell_tag(c[0], c[1], c[2]);
         // chained spatial hash: push onto the list of bucket hash(cell) -- one atomic exchange;
         // heads hold index + 1 (0 = empty bucket)
@@ -269,7 +306,7 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
         const uint32_t prev = atomicExch(tab.bits + (size_t)s * tab.bwords + b,
                                          (tag << kEpochShift) | ((uint32_t)r + 1u));
         next = ((prev >> kEpochShift) == tag && (prev & kIdxMask)) ? (prev & kIdxMask) - 1u : kNil;
-    } else if (!kChained && cell_of(g, p, c)) {
+    } else if (kGrid == kOpen && cell_of(g, p, c)) {
         const unsigned long long key = pack_key(c[0], c[1], c[2]);
         const uint32_t hb = bit_hash(c[0], c[1], c[2]) & tab.bmask;
         atomicOr(tab.bits + (size_t)s * tab.bwords + (hb >> 5), 1u << (hb & 31));
@@ -565,6 +602,166 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
 }
 
 // ---------------------------------------------------------------------------------------
+// CSR grid (kCsr, sort + segment): after the build counted every object into its cell's slot,
+// k_csr_alloc gives each occupied slot a segment [start, start + count) of the step's entry array
+// (warp prefix sums, one atomic per warp) and k_csr_scatter moves each object's entry to
+// start + rank: the objects of a cell are contiguous, ordered by cell.  The scan then runs one
+// thread per segment position -- the objects of a cell are adjacent lanes probing the same
+// neighbour slots -- and reads each neighbour cell as one contiguous range (independent loads
+// instead of a linked list's dependent ones).
+// ---------------------------------------------------------------------------------------
+__global__ void k_csr_alloc(const Slot* __restrict__ slots, uint32_t* __restrict__ start, uint64_t M,
+                            int B, uint32_t tag, unsigned long long* __restrict__ total)
+{
+    const uint64_t gi = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const int s = (int)(gi / M);
+    const uint64_t h = gi - (uint64_t)s * M;
+    const bool in = s < B;
+    uint32_t cnt = 0;
+    if (in) {
+        const unsigned long long w1 = slots[(size_t)s * M + h].head;
+        cnt = (uint32_t)(w1 >> 32) == tag ? (uint32_t)w1 : 0u;
+    }
+    // warp inclusive prefix sum (the warp's slots all belong to one step: M is a multiple of 32)
+    const unsigned lane = threadIdx.x & 31;
+    uint32_t inc = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= (unsigned)o) inc += y;
+    }
+    unsigned long long base = 0;
+    if (lane == 31 && in && inc) base = atomicAdd(total + s, (unsigned long long)inc);
+    base = __shfl_sync(0xffffffffu, base, 31);
+    if (in) start[(size_t)s * M + h] = (uint32_t)base + inc - cnt;
+}
+
+__global__ void k_csr_scatter(const Entry* __restrict__ tmp, const Slot* __restrict__ slots,
+                              const uint32_t* __restrict__ start, uint64_t M, int64_t n, int B,
+                              Entry* __restrict__ csr)
+{
+    const int64_t gi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int s = (int)(gi / n);
+    const int64_t r = gi - (int64_t)s * n;
+    if (s >= B) return;
+    Entry e = tmp[(size_t)s * n + r];
+    if (e.next == kNil) return;   // out of the key range (CD_ERANGE already raised)
+    const size_t sh = (size_t)s * M + e.next;
+    const uint32_t st = start[sh];
+    const uint32_t cnt = (uint32_t)slots[sh].head;
+    const uint32_t pos = st + e.tag;
+    e.next = (uint32_t)r;      // the object
+    e.tag = st + cnt;          // end of its cell's segment
+    csr[(size_t)s * n + pos] = e;
+}
+
+cudaError_t launch_csr_segments(const Slot* slots, uint32_t* start, uint64_t M, const Entry* tmp,
+                                Entry* csr, int64_t n, int B, uint32_t tag, unsigned long long* total,
+                                cudaStream_t st, LaunchCount& lc)
+{
+    if (B <= 0) return cudaSuccess;
+    cudaError_t e = cudaMemsetAsync(total, 0, sizeof(unsigned long long) * (size_t)B, st);
+    if (e != cudaSuccess) return e;
+    k_csr_alloc<<<blocks_for((int64_t)(M * (uint64_t)B), 256), 256, 0, st>>>(slots, start, M, B, tag, total);
+    lc.bump();
+    k_csr_scatter<<<blocks_for(n * B, 256), 256, 0, st>>>(tmp, slots, start, M, n, B, csr);
+    lc.bump();
+    return cudaGetLastError();
+}
+
+// Look a cell up in the CSR slot table: its segment [*st, *st + *cnt), false if empty.
+__device__ __forceinline__ bool csr_find(const Slot* __restrict__ slots, const uint32_t* __restrict__ start,
+                                         uint64_t mask, unsigned long long key, uint32_t tag,
+                                         uint32_t* st, uint32_t* cnt)
+{
+    uint64_t h = fmix64(key) & mask;
+    while (true) {
+        const ulonglong2 w = __ldg(reinterpret_cast<const ulonglong2*>(slots + h));
+        if ((uint32_t)(w.y >> 32) != tag) return false;
+        if (w.x == key) {
+            *cnt = (uint32_t)w.y;
+            *st = __ldg(start + h);
+            return true;
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+__device__ __forceinline__ void csr_range(const GridGeom& g, const Entry* __restrict__ C, uint32_t u,
+                                          uint32_t end, uint32_t id, const double p[3], uint32_t step,
+                                          Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
+{
+#pragma unroll 4
+    for (; u < end; ++u) {
+        const Entry e = C[u];
+        test_pair(g, id, e.next, p, e, step, q, qcap, ctrl);
+    }
+}
+
+__device__ __forceinline__ void do_scan_csr(const GridGeom& g, const GridTab& tab,
+                                            const uint32_t* __restrict__ starts, const Entry* __restrict__ csr,
+                                            int64_t n, uint64_t mask, int64_t k0, int s, int64_t t,
+                                            uint32_t tag, Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
+{
+    const Slot* slots = tab.slots + (size_t)s * (mask + 1);
+    const uint32_t* start = starts + (size_t)s * (mask + 1);
+    const uint32_t* bits = tab.bits + (size_t)s * tab.bwords;
+    const uint32_t bmask = tab.bmask;
+    const Entry* C = csr + (size_t)s * n;
+    const uint32_t step = (uint32_t)(k0 + s);
+    const Entry me = C[t];
+    const double p[3] = {me.x, me.y, me.z};
+    int c[3];
+    double fr[3];
+    if (!cell_of(g, p, c, fr)) return;
+    // (1) own cell: the later positions of the segment, each pair once
+    csr_range(g, C, (uint32_t)t + 1, me.tag, me.next, p, step, q, qcap, ctrl);
+    // (2) other cells: half-shell (L < 2 g_c) or the positive half-space of the ball (L >= 2 g_c)
+    const uint32_t hx0 = (uint32_t)c[0] * kHX, hy0 = (uint32_t)c[1] * kHY, hz0 = (uint32_t)c[2] * kHZ;
+    uint32_t st, cnt;
+    if (g.halfshell) {
+        uint32_t hit = 0;
+#pragma unroll
+        for (int o = 1; o < 14; ++o) {
+            const uint32_t hb = bit_mix((hx0 + (uint32_t)kHalfShell[o][0] * kHX) ^
+                                        (hy0 + (uint32_t)kHalfShell[o][1] * kHY) ^
+                                        (hz0 + (uint32_t)kHalfShell[o][2] * kHZ)) & bmask;
+            hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << o;
+        }
+        while (hit) {
+            const int o = __ffs(hit) - 1;
+            hit &= hit - 1;
+            if (csr_find(slots, start, mask, pack_key(c[0] + kHalfShell[o][0], c[1] + kHalfShell[o][1],
+                                                      c[2] + kHalfShell[o][2]), tag, &st, &cnt))
+                csr_range(g, C, st, st + cnt, me.next, p, step, q, qcap, ctrl);
+        }
+    } else {
+        const double rl = g.reach * g.inv_cell;
+        const int d0 = fr[0] < rl ? -1 : (fr[0] > 1.0 - rl ? 1 : 0);
+        const int d1 = fr[1] < rl ? -1 : (fr[1] > 1.0 - rl ? 1 : 0);
+        const int d2 = fr[2] < rl ? -1 : (fr[2] > 1.0 - rl ? 1 : 0);
+        const uint32_t hx1 = hx0 + (uint32_t)d0 * kHX, hy1 = hy0 + (uint32_t)d1 * kHY,
+                       hz1 = hz0 + (uint32_t)d2 * kHZ;
+        const uint32_t pos = (d0 > 0 ? 0xAAu : 0u) | (d1 > 0 ? 0x44u : 0u) | (d2 > 0 ? 0x10u : 0u);
+        const uint32_t valid = (d0 ? 0xFFu : 0x55u) & (d1 ? 0xFFu : 0x33u) & (d2 ? 0xFFu : 0x0Fu) & pos;
+        uint32_t hit = 0;
+#pragma unroll
+        for (int b = 1; b < 8; ++b) {
+            const uint32_t hb = bit_mix(((b & 1) ? hx1 : hx0) ^ ((b & 2) ? hy1 : hy0) ^
+                                        ((b & 4) ? hz1 : hz0)) & bmask;
+            if ((valid >> b) & 1u) hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << b;
+        }
+        while (hit) {
+            const int b = __ffs(hit) - 1;
+            hit &= hit - 1;
+            if (csr_find(slots, start, mask, pack_key(c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0),
+                                                      c[2] + ((b & 4) ? d2 : 0)), tag, &st, &cnt))
+                csr_range(g, C, st, st + cnt, me.next, p, step, q, qcap, ctrl);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------
 // One launch per batch (horizontal fusion): blocks of three roles run side by side, so the
 // latency-bound build (fp64 Contour + atomics) and scan (probes) hide each other's stalls.
 //   role A: build batch b + 1, class-0 objects     (slot set (b+1) % 2, bitmap set (b+1) % 3)
@@ -578,8 +775,8 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
 #ifndef CD_OPEN_MINB
 #define CD_OPEN_MINB 6
 #endif
-template <bool kChained, int kJ2>
-__global__ void __launch_bounds__(256, kChained ? CD_STEP_MINB : CD_OPEN_MINB) k_step(StepArgs a)
+template <int kGrid, int kJ2>
+__global__ void __launch_bounds__(256, kGrid == kChained ? CD_STEP_MINB : CD_OPEN_MINB) k_step(StepArgs a)
 {
     const uint32_t bx = blockIdx.x;
     const uint32_t nbA = (uint32_t)a.nbA, nbB = (uint32_t)a.nbB, nbC = (uint32_t)a.nbC;
@@ -594,14 +791,14 @@ __global__ void __launch_bounds__(256, kChained ? CD_STEP_MINB : CD_OPEN_MINB) k
         const int s = (int)(bx / nbA);
         const int64_t r = (int64_t)(bx % nbA) * 256 + threadIdx.x;
         if (r < a.O.n0)
-            do_build<true, kChained, kJ2>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
+            do_build<true, kGrid, kJ2>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
                                      a.dt, a.build_tag, a.ctrl);
     } else if (bx < nA + nB) {
         const uint32_t b2 = bx - nA;
         const int s = (int)(b2 / nbB);
         const int64_t r = a.O.n0 + (int64_t)(b2 % nbB) * 256 + threadIdx.x;
         if (r < a.O.n)
-            do_build<false, kChained, kJ2>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
+            do_build<false, kGrid, kJ2>(a.O, a.g, a.build_tab, a.build_ents, a.mask, a.build_k0, s, r, a.t0,
                                       a.dt, a.build_tag, a.ctrl);
     } else {
         const uint32_t b3 = bx - nA - nB;
@@ -612,7 +809,7 @@ __global__ void __launch_bounds__(256, kChained ? CD_STEP_MINB : CD_OPEN_MINB) k
         const int64_t nth = a.nCblocks * 256;
         const int64_t nw4 = (int64_t)a.zero_depth * a.zero_bits_words / 4;
         uint4* zb = reinterpret_cast<uint4*>(a.zero_bits);
-        if (!kChained)   // chained heads are epoch-tagged: nothing to clear
+        if (kGrid != kChained)   // chained heads are epoch-tagged: nothing to clear
             for (int64_t i = tid; i < nw4; i += nth) zb[i] = make_uint4(0u, 0u, 0u, 0u);
         if (a.scan_B == 0) return;
         const int s = (int)(b3 / nbC);
@@ -624,9 +821,12 @@ __global__ void __launch_bounds__(256, kChained ? CD_STEP_MINB : CD_OPEN_MINB) k
             __syncwarp();
         }
         if (r < a.O.n) {
-            if (kChained)
+            if (kGrid == kChained)
                 do_scan_chained(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
                                 a.qcap, a.ctrl);
+            else if (kGrid == kCsr)
+                do_scan_csr(a.g, a.scan_tab, a.scan_start, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r,
+                            a.scan_tag, a.q, a.qcap, a.ctrl);
             else
                 do_scan(a.g, a.scan_tab, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r, a.scan_tag, a.q,
                         a.qcap, a.ctrl);
@@ -659,12 +859,16 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
     const size_t smem = a.g.stage ? sizeof(Cand) * kSCand : 0;   // candidate staging buffer
     if (a.O.j2) {   // J2 secular propagator: the rotation is compiled into its own instances
         if (a.chained)
-            return launch_ex(k_step<true, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, a.pdl != 0, a);
-        return launch_ex(k_step<false, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
+            return launch_ex(k_step<kChained, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, a.pdl != 0, a);
+        if (a.csr)
+            return launch_ex(k_step<kCsr, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
+        return launch_ex(k_step<kOpen, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
     }
     if (a.chained)
-        return launch_ex(k_step<true, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, a.pdl != 0, a);
-    return launch_ex(k_step<false, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
+        return launch_ex(k_step<kChained, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, a.pdl != 0, a);
+    if (a.csr)
+        return launch_ex(k_step<kCsr, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
+    return launch_ex(k_step<kOpen, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
 }
 
 // ---------------------------------------------------------------------------------------

@@ -100,7 +100,9 @@ def test_candidates_ragged_sizes(n, steps, d):
                                 dict(grid_table=2, cell_factor=1.0), dict(grid_table=1, round_steps=5),
                                 dict(cell_factor=2.0), dict(cell_factor=1.5, grid_origin=(-3e3, 7.5, 1e4)),
                                 dict(cell_factor=3.7), dict(batch_object_steps=1),
-                                dict(round_steps=7), dict(batch_object_steps=10 ** 7)])
+                                dict(round_steps=7), dict(batch_object_steps=10 ** 7),
+                                dict(grid_table=3), dict(grid_table=3, cell_factor=1.0),
+                                dict(grid_table=3, batch_object_steps=1), dict(grid_table=3, round_steps=5)])
 def test_candidates_invariance(kw):
     pop = _mix(8000, 5)
     d = 20.0
