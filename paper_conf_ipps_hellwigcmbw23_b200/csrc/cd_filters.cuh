@@ -17,7 +17,7 @@ constexpr double kTwoPiH = 6.28318530717958647692;
 struct __align__(128) HOrbit {   // one 128-byte line per object (compact gather in the filter)
     double e, q, Q, p, nm, M0;
     double P[3], Qv[3], h[3];
-    double pad;
+    double inm;   // 1 / nm
 };
 static_assert(sizeof(HOrbit) == 128, "HOrbit must be one 128-byte line");
 
@@ -40,9 +40,11 @@ __device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o)
     o.p = a * (1.0 - o.e) * (1.0 + o.e);
     o.nm = O.at(kNm, r);
     o.M0 = O.at(kM0, r);
-    o.pad = 0.0;
+    o.inm = 1.0 / o.nm;
 }
 
+// Divisions are reciprocal estimates refined to full precision (rcp_fast: two Newton steps) times
+// the numerator -- the filters' decisions have km margins, 2 roundings instead of 1 are immaterial.
 // Node geometry of one orbit of a pair (reading R17), all algebraic: the mutual node line is a
 // unit vector in the orbit plane, so its components along P and Q are the cosine and sine of its
 // true anomaly f; the window half-angle a = asin(s) has sin a = s, cos a = sqrt(1 - s^2).  The
@@ -58,7 +60,7 @@ __device__ __forceinline__ double mean_of_true_cs(double c, double s, double e)
 {
     const double w = sqrt((1.0 - e) * (1.0 + e));
     const double E = atan2(w * s, e + c);
-    return E - e * (w * s / fma(e, c, 1.0));
+    return E - e * (w * s * rcp_fast(fma(e, c, 1.0)));
 }
 
 // radius range over the true anomalies (f - a, f + a) of node `sg` (+1: f, -1: f + pi), a < pi/2:
@@ -69,7 +71,7 @@ __device__ __forceinline__ void radius_range(const HOrbit& o, const NodeGeom& g,
 {
     const double cf = sg * g.cf, sf = sg * g.sf;
     const double c1 = fma(cf, g.ca, sf * g.sa), c2 = fma(cf, g.ca, -sf * g.sa);
-    const double r1 = o.p / fma(o.e, c1, 1.0), r2 = o.p / fma(o.e, c2, 1.0);
+    const double r1 = o.p * rcp_fast(fma(o.e, c1, 1.0)), r2 = o.p * rcp_fast(fma(o.e, c2, 1.0));
     rmin = fmin(r1, r2);
     rmax = fmax(r1, r2);
     if (cf >= g.ca) rmin = o.q;    // perigee inside
@@ -84,8 +86,8 @@ __device__ __forceinline__ void node_window(const HOrbit& o, const NodeGeom& g, 
     const double Ml = mean_of_true_cs(fma(cf, g.ca, sf * g.sa), fma(sf, g.ca, -cf * g.sa), o.e);
     double Mh = mean_of_true_cs(fma(cf, g.ca, -sf * g.sa), fma(sf, g.ca, cf * g.sa), o.e);
     if (Mh < Ml) Mh += kTwoPiH;
-    tl = (Ml - o.M0) / o.nm;
-    th = (Mh - o.M0) / o.nm;
+    tl = (Ml - o.M0) * o.inm;
+    th = (Mh - o.M0) * o.inm;
 }
 
 // Pair geometry of the filter chain (reading R17).  Returns 1 if the apogee/perigee filter
@@ -100,8 +102,8 @@ __device__ __forceinline__ int pair_geometry(const HOrbit& A, const HOrbit& B, d
     const double c[3] = {A.h[1] * B.h[2] - A.h[2] * B.h[1], A.h[2] * B.h[0] - A.h[0] * B.h[2],
                          A.h[0] * B.h[1] - A.h[1] * B.h[0]};
     const double sD = sqrt(c[0] * c[0] + c[1] * c[1] + c[2] * c[2]);
-    const double sA = sD > 0.0 ? d / (A.q * sD) : 2.0;
-    const double sB = sD > 0.0 ? d / (B.q * sD) : 2.0;
+    const double sA = sD > 0.0 ? d * rcp_fast(A.q * sD) : 2.0;
+    const double sB = sD > 0.0 ? d * rcp_fast(B.q * sD) : 2.0;
     coplanar = sA >= 1.0 || sB >= 1.0;
     if (coplanar) return 0;
     gA.sa = sA;
@@ -110,15 +112,16 @@ __device__ __forceinline__ int pair_geometry(const HOrbit& A, const HOrbit& B, d
     gB.ca = sqrt((1.0 - sB) * (1.0 + sB));
     coplanar = A.q * gA.ca + B.q * gB.ca <= d;
     if (coplanar) return 0;
-    const double nn[3] = {c[0] / sD, c[1] / sD, c[2] / sD};
+    const double isD = rcp_fast(sD);
+    const double nn[3] = {c[0] * isD, c[1] * isD, c[2] * isD};
     double x = nn[0] * A.P[0] + nn[1] * A.P[1] + nn[2] * A.P[2];
     double y = nn[0] * A.Qv[0] + nn[1] * A.Qv[1] + nn[2] * A.Qv[2];
-    double k = 1.0 / sqrt(x * x + y * y);
+    double k = rcp_fast(sqrt(x * x + y * y));
     gA.cf = x * k;
     gA.sf = y * k;
     x = nn[0] * B.P[0] + nn[1] * B.P[1] + nn[2] * B.P[2];
     y = nn[0] * B.Qv[0] + nn[1] * B.Qv[1] + nn[2] * B.Qv[2];
-    k = 1.0 / sqrt(x * x + y * y);
+    k = rcp_fast(sqrt(x * x + y * y));
     gB.cf = x * k;
     gB.sf = y * k;
     return 0;

@@ -88,14 +88,14 @@ __global__ void __launch_bounds__(256, CD_FILTER_MINB) k_hybrid_filter(Orbits O,
             // computed when one of A's copies meets the cell (most pairs end here)
             double atl, ath, btl, bth;
             node_window(A, gA, sg, atl, ath);
-            const double TA = kTwoPiH / A.nm, TB = kTwoPiH / B.nm;
-            const double ka = floor((lo - (ath - tk)) / TA);
+            const double TA = kTwoPiH * A.inm, TB = kTwoPiH * B.inm;
+            const double ka = floor((lo - (ath - tk)) * (A.nm * (1.0 / kTwoPiH)));
             bool a_meets = false;
             for (int x = 0; x < 3; ++x)
                 a_meets = a_meets || fmin(ath - tk + (ka + x) * TA, hi) >= fmax(atl - tk + (ka + x) * TA, lo);
             if (!a_meets) continue;
             node_window(B, gB, sg, btl, bth);
-            const double kb = floor((lo - (bth - tk)) / TB);
+            const double kb = floor((lo - (bth - tk)) * (B.nm * (1.0 / kTwoPiH)));
             for (int x = 0; x < 3; ++x) {
                 const double al = fmax(atl - tk + (ka + x) * TA, lo), ah = fmin(ath - tk + (ka + x) * TA, hi);
                 if (!(ah >= al)) continue;
