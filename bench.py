@@ -103,6 +103,24 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
+def cpu_model():
+    """The host CPU (lscpu "Model name"), for the cpu_baseline record."""
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name:"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    try:
+        for line in Path("/proc/cpuinfo").read_text().splitlines():
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
 def population(args):
     from tools import popgen
     pop, cfg, _ = popgen.make_config(args.config, n=args.n)
@@ -147,7 +165,7 @@ def run_reference(args):
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "config": workload_config(args, cfg, n, dt, K),
             "cpu_baseline": {"value": value, "unit": "object-steps/s", "cores": threads,
-                             "kind": "oracle",
+                             "kind": "oracle", "cpu_model": cpu_model(),
                              "sample": f"{per} consecutive {dt:g}-s steps of the 24 h window per "
                                        f"bench step (CPU grid + conjunctions), {n} objects"},
             "e2e": {"value": value, "unit": "object-steps/s", "h2d_bytes_per_step": 0,
@@ -427,6 +445,7 @@ def run_ours(args):
         per = args.cpu_steps
         sec, threads = cpu_oracle_sample(pop, cfg, dt, cfg.d, k0, per)
         cpu = {"value": n * per / sec, "unit": "object-steps/s", "cores": threads, "kind": "oracle",
+               "cpu_model": cpu_model(),
                "sample": f"steps [{k0}, {k0 + per}) of the same 24 h window ({per} x {n} "
                          f"object-steps: CPU grid candidates + conjunctions), {sec:.1f} s"}
 
