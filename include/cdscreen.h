@@ -155,6 +155,12 @@ typedef struct {
                                   (e.g. the next time slice) skips that call's density-probe round */
     int grid_table;            /* the grid structure the call used: 1 open addressing, 2 chained,
                                   3 CSR (sort + segment)                                          */
+    uint64_t grids_in_flight;  /* B: sampling steps per in-flight batch (the paper's p grids,
+                                  P:236-252): min(batch_object_steps / n, what free memory holds) */
+    uint64_t raw_pairs;        /* emit_raw_counts: pairs the scan examined (before the distance
+                                  test); with cell_factor = 1 and grid_table = 1 this is the
+                                  paper's count of object pairs in the same or neighbouring cells
+                                  (each unordered pair once per step)                */
 } cd_stats;
 
 typedef struct {
@@ -222,6 +228,9 @@ typedef struct {
                                  (results do not depend on it).  0 = auto (default: every
                                  max(16, 64 s / dt) steps for >= 4M objects in CD_GRID, else
                                  off), < 0 = off, R > 0 = every R steps                         */
+    int emit_raw_counts;      /* also count the pairs the scan examines into cd_stats.raw_pairs
+                                 (the paper's raw count with cell_factor = 1, grid_table = 1;
+                                 P:95); default 0                                   */
 } cd_options;
 
 /* Fill *opt with the defaults above. */

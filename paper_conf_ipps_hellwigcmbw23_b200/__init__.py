@@ -75,7 +75,8 @@ class cd_stats(C.Structure):
                 ("ms_precompute", C.c_double), ("launches_clear", C.c_uint64),
                 ("launches_propagate", C.c_uint64), ("launches_insert", C.c_uint64),
                 ("launches_scan", C.c_uint64), ("launches_refine", C.c_uint64),
-                ("step_launches", C.c_uint64), ("cell_factor", C.c_double), ("grid_table", C.c_int)]
+                ("step_launches", C.c_uint64), ("cell_factor", C.c_double), ("grid_table", C.c_int),
+                ("grids_in_flight", C.c_uint64), ("raw_pairs", C.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -95,7 +96,7 @@ class cd_options(C.Structure):
                 ("stats", C.POINTER(cd_stats)), ("propagator", C.c_int),
                 ("shell_lo", C.c_double), ("shell_hi", C.c_double),
                 ("alloc", ALLOC_FN), ("free", FREE_FN), ("alloc_ctx", C.c_void_p),
-                ("shards", C.c_int), ("resort_steps", C.c_int)]
+                ("shards", C.c_int), ("resort_steps", C.c_int), ("emit_raw_counts", C.c_int)]
 
 
 class cd_plan_info(C.Structure):
@@ -314,7 +315,7 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
                  cell_factor=None, batch_object_steps=None, round_steps=None,
                  outputs_on_device=False, inputs_on_device=False, profile_phases=False,
                  l2_persist=None, grid_table=None, propagator=None, shell=None, allocator=None,
-                 shards=None, kepler_points=None, resort_steps=None):
+                 shards=None, kepler_points=None, resort_steps=None, emit_raw_counts=False):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -359,6 +360,7 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
         o.kepler_points = int(kepler_points)
     if resort_steps is not None:
         o.resort_steps = int(resort_steps)
+    o.emit_raw_counts = int(bool(emit_raw_counts))
     return o
 
 

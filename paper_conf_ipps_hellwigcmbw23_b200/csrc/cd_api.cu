@@ -742,6 +742,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     g.band_lo2 = o.shell_hi > 0.0 ? o.shell_lo * o.shell_lo : 0.0;
     g.band_hi2 = o.shell_hi > 0.0 ? o.shell_hi * o.shell_hi : HUGE_VAL;
     g.sig = nullptr;
+    g.raw = o.emit_raw_counts ? 1 : 0;
     RefineParams P{t0, t1, dt, d, gc, nullptr};
 
     R.cand.st = st;
@@ -772,6 +773,27 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     const uint64_t chain_words = can_chain ? std::max<uint64_t>(next_pow2((uint64_t)n * CD_CHAIN_FACTOR), 1024) : 0;
     const uint64_t nbits = std::max<uint64_t>(next_pow2((uint64_t)n * 32), 1024);   // open: >= 32 bits/object
     const uint32_t bwords = (uint32_t)std::max<uint64_t>(chain_words, can_open ? nbits / 32 : 0);
+    // memory-bounded grids in flight (p = (m - a_s - a_k - a_ch) / (a_gh + a_l)): a
+    // batch of B steps holds B grids in each rotating set (2 slot sets, 3 bitmap / head sets, 3
+    // entry sets, CSR scratch); B never exceeds what the free device memory holds, keeping an
+    // eighth and 256 MB back for queues, sort scratch and results.  (On a 180 GB B200 the default
+    // batch, 2^20 object-steps, is the binding limit up to ~10^8 objects.)
+    {
+        size_t fr = 0, tot = 0;
+        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) {
+            const double per = (can_open ? 2.0 * sizeof(Slot) * (double)M : 0.0) + 3.0 * 4.0 * (double)bwords +
+                               3.0 * sizeof(Entry) * (double)n +
+                               (csr ? sizeof(Entry) * (double)n + 2.0 * 4.0 * (double)M : 0.0);
+            const double avail = (double)fr * 0.875 - 256e6;
+            const int64_t p = avail > 0.0 ? (int64_t)(avail / per) : 0;
+            if (p < 1)
+                return fail(CD_ENOMEM, "one step's grid (%.3g GB per rotating set) does not fit the free device memory (%.3g GB)",
+                            per / 1e9, (double)fr / 1e9);
+            Bmax = std::min<int64_t>(Bmax, p);
+        }
+        cudaGetLastError();
+    }
+    stats.grids_in_flight = (uint64_t)Bmax;
     const size_t slot_bytes = can_open ? sizeof(Slot) * (size_t)Bmax * M : 0;
     auto pick_chained = [&](const GridGeom& gg) {
         if (n > (int64_t)kMaxChainN) return false;   // 24-bit head indices
@@ -961,6 +983,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     int nin = 0, next_slot = 0;
     auto enqueue_round = [&](int64_t kr, int64_t Rk, int slot) -> cd_status {
         CU(cudaMemsetAsync(&ctrl.p->n_cand, 0, sizeof(unsigned long long), st));
+        CU(cudaMemsetAsync(&ctrl.p->n_raw, 0, sizeof(unsigned long long), st));
         CU(cudaMemsetAsync(nwork.p, 0, sizeof(unsigned long long), st));
         // software pipeline over the round's batches: launch i builds batch i and scans i - 1
         const int64_t J = (Rk + Bmax - 1) / Bmax;
@@ -1115,6 +1138,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             back.n_path = hyb_before[2];
             back.n_time = hyb_before[3];
             back.n_cand = 0;
+            back.n_raw = 0;
             back.err_range = 0;
             back.err_internal = 0;
             Ctrl* stage = hslot[rd.slot];
@@ -1126,6 +1150,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         }
         // round accepted
         stats.candidates += hctrl->n_cand;
+        stats.raw_pairs += hctrl->n_raw;
         stats.refined += hnwork;
         if (want == Want::Cand && hctrl->n_cand) {
             if (R.n_cand + hctrl->n_cand > ccap) {
@@ -1367,6 +1392,7 @@ cd_status screen_sharded(Call& C, const cd_elements* el, size_t n, double t0, do
         memset(&ss, 0, sizeof ss);
         TRY(run(C, Ss, t0, t1, dt, d, mode, os, K, Want::Conj, Rs, ss));
         stats.candidates += ss.candidates;
+        stats.raw_pairs += ss.raw_pairs;
         stats.refined += ss.refined;
         stats.retries += ss.retries;
         stats.hybrid_ap_rejected += ss.hybrid_ap_rejected;

@@ -419,6 +419,7 @@ struct GridGeom {
     // spatial slot order: entry index (slot) -> internal object id of the scanned batch
     // (nullptr: slots are internal ids)
     const uint32_t* sig;
+    int raw;             // cd_options.emit_raw_counts: count every pair examined (Ctrl::n_raw)
 };
 
 // Cell of position p: c = floor((p - o) / L) per axis (R7); frac = (p - o)/L - c in [0, 1).
@@ -582,6 +583,7 @@ struct Ctrl {   // device-side counters and flags of one call
     unsigned long long n_ap, n_coplanar, n_path, n_time;
     int err_range;
     int err_internal;
+    unsigned long long n_raw;   // pairs examined by the scan (emit_raw_counts; per round)
 };
 
 }  // namespace cdk

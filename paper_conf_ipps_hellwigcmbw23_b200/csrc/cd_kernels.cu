@@ -355,11 +355,13 @@ constexpr unsigned kSCand = 1024;              // per block (256 threads)
 constexpr unsigned kSWarp = kSCand / 8;        // per warp
 extern __shared__ Cand s_cand[];
 __shared__ unsigned s_nw[8];
+__shared__ unsigned s_rw[8];   // per warp: pairs examined (emit_raw_counts)
 
 __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_t j, const double p[3],
                                           const Entry& ej, uint32_t step, Cand* __restrict__ q,
                                           size_t qcap, Ctrl* ctrl)
 {
+    if (g.raw) atomicAdd(&s_rw[threadIdx.x >> 5], 1u);
     const double dx = p[0] - ej.x, dy = p[1] - ej.y, dz = p[2] - ej.z;
     if (fma(dx, dx, fma(dy, dy, dz * dz)) < g.gc2) {
         // radial shard: the pair belongs to the shard holding the smaller radius (identical
@@ -816,8 +818,11 @@ __global__ void __launch_bounds__(256, kGrid == kChained ? CD_STEP_MINB : CD_OPE
         const int64_t r = (int64_t)(b3 % nbC) * 256 + threadIdx.x;
         const bool stage = a.g.stage != 0;   // uniform over the launch
         const unsigned lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-        if (stage) {
-            if (lane == 0) s_nw[wid] = 0;
+        if (stage || a.g.raw) {
+            if (lane == 0) {
+                s_nw[wid] = 0;
+                s_rw[wid] = 0;
+            }
             __syncwarp();
         }
         if (r < a.O.n) {
@@ -830,6 +835,10 @@ __global__ void __launch_bounds__(256, kGrid == kChained ? CD_STEP_MINB : CD_OPE
             else
                 do_scan(a.g, a.scan_tab, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r, a.scan_tag, a.q,
                         a.qcap, a.ctrl);
+        }
+        if (a.g.raw) {
+            __syncwarp();
+            if (lane == 0 && s_rw[wid]) atomicAdd(&a.ctrl->n_raw, (unsigned long long)s_rw[wid]);
         }
         if (!stage) return;
         // flush the warp's staged candidates: one global atomic, coalesced copy

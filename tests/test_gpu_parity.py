@@ -305,3 +305,28 @@ def test_spatial_resort_is_invisible(mode, dt, R):
         parity.compare_candidates(pop, K1, Ko, t0, dt, gc)
         Co = oracle.conjunctions(pop, t0, t1, dt, d, gc, Ko)
         parity.compare_conjunctions(pop, C1, Co, t0, t1, dt, d, gc)
+
+
+def test_raw_counts_and_grids_in_flight():
+    """emit_raw_counts with the paper's cell (cell_factor 1) and map (grid_table 1): raw_pairs is
+    the number of object pairs in the same or neighbouring cells of edge g_c, each unordered pair
+    once per step -- counted here by brute force from the oracle's positions.
+    grids_in_flight reports the batch B (the paper's p)."""
+    pop = _mix(3000, 41, "paper", 500)
+    d, dt, t0, t1 = 30.0, 1.0, 0.0, 9.0
+    gc = oracle.cell_size(d, dt)
+    K, st = cds.candidates(pop, t0, t1, dt, d, cell_factor=1.0, grid_table=1, emit_raw_counts=True,
+                           return_stats=True)
+    want = 0
+    x = oracle.propagate(pop, t0 + dt * np.arange(10))
+    # the library's cell edge for cell_factor 1 is g_c (1 + 1e-12), origin 0
+    L = gc * (1.0 + 1e-12)
+    for q in range(10):
+        c = np.floor(x[q] / L).astype(np.int64)
+        diff = np.abs(c[:, None, :] - c[None, :, :]).max(axis=2)
+        want += int(np.count_nonzero(np.triu(diff <= 1, 1)))
+    assert st["raw_pairs"] == want, (st["raw_pairs"], want)
+    assert st["raw_pairs"] > len(K) > 0
+    assert st["grids_in_flight"] >= 1
+    _, st2 = cds.candidates(pop, t0, t1, dt, d, return_stats=True)
+    assert st2["raw_pairs"] == 0
