@@ -397,7 +397,7 @@ def run_ours(args):
         torch.cuda.synchronize()
         e2e_ms.append(e0.elapsed_time(e1))
     ne2e = len(e2e_ms)
-    e2e_tot = float(np.sum(e2e_ms))
+    e2e_tot = max(float(np.sum(e2e_ms)), 1e-9)
     if distributed:
         t = torch.tensor([e2e_tot], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -405,7 +405,7 @@ def run_ours(args):
     e2e_units = float(n) * (K / S) * ne2e * world
     e2e = {"value": e2e_units / (e2e_tot / 1e3), "unit": "object-steps/s",
            "h2d_bytes_per_step": 48 * n, "d2h_bytes_per_step": int(d2h / max(1, ne2e)),
-           "steps": ne2e}
+           "steps": ne2e} if ne2e else None
 
     if rank != 0:
         if distributed:

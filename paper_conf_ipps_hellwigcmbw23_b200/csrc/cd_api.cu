@@ -779,11 +779,12 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     // eighth and 256 MB back for queues, sort scratch and results.  (On a 180 GB B200 the default
     // batch, 2^20 object-steps, is the binding limit up to ~10^8 objects.)
     {
+        const double per = (can_open ? 2.0 * sizeof(Slot) * (double)M : 0.0) + 3.0 * 4.0 * (double)bwords +
+                           3.0 * sizeof(Entry) * (double)n +
+                           (csr ? sizeof(Entry) * (double)n + 2.0 * 4.0 * (double)M : 0.0);
         size_t fr = 0, tot = 0;
-        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) {
-            const double per = (can_open ? 2.0 * sizeof(Slot) * (double)M : 0.0) + 3.0 * 4.0 * (double)bwords +
-                               3.0 * sizeof(Entry) * (double)n +
-                               (csr ? sizeof(Entry) * (double)n + 2.0 * 4.0 * (double)M : 0.0);
+        // the free-memory query costs a driver call: only when the batch could come near it
+        if (per * (double)Bmax > 4e9 && cudaMemGetInfo(&fr, &tot) == cudaSuccess) {
             const double avail = (double)fr * 0.875 - 256e6;
             const int64_t p = avail > 0.0 ? (int64_t)(avail / per) : 0;
             if (p < 1)
@@ -1678,6 +1679,14 @@ cd_status cd_conjunctions_sort_device(cd_conjunction* data, size_t n, void* stre
         if (n == 0) return CD_OK;
         if (!data) return fail(CD_EINVAL, "data must be non-NULL");
         cudaStream_t st = (cudaStream_t)stream;
+        // scratch from the library's private pool of the current device (which keeps its memory:
+        // the device's default pool would unmap and remap it on every merge)
+        int dev = 0;
+        CU(cudaGetDevice(&dev));
+        struct PoolScope {
+            explicit PoolScope(cudaMemPool_t p) { g_pool = p; }
+            ~PoolScope() { g_pool = nullptr; }
+        } scope(setup_pool(dev));
         LaunchCount lc;
         DBuf<Conj> tmp(st);
         CU(tmp.alloc(n));

@@ -92,9 +92,17 @@ def device_records_to_tensor(out, device):
 
 
 def records_to_numpy(t):
+    """Host copy of a record tensor (m, 32) as a CONJ_DTYPE array (one D2H copy into pinned
+    memory, then a view -- no further copies)."""
+    import torch
     from . import CONJ_DTYPE
-    a = t.cpu().numpy()
-    return np.frombuffer(a.tobytes(), dtype=CONJ_DTYPE).copy()
+    if t.is_cuda:
+        h = torch.empty(t.shape, dtype=torch.uint8, pin_memory=True)
+        h.copy_(t)
+        a = h.numpy()
+    else:
+        a = t.contiguous().numpy()
+    return a.reshape(-1).view(CONJ_DTYPE)
 
 
 FAR_KM = 1.0e9   # upper bound of the outermost shard (cd_options.shell_hi must be finite)
