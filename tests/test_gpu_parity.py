@@ -330,3 +330,22 @@ def test_raw_counts_and_grids_in_flight():
     assert st["grids_in_flight"] >= 1
     _, st2 = cds.candidates(pop, t0, t1, dt, d, return_stats=True)
     assert st2["raw_pairs"] == 0
+
+
+def test_memory_bounded_batch():
+    """the number of grids in flight p is bounded by the free device memory.  With a
+    huge requested batch and most of the device memory taken, the call still runs, with fewer
+    steps per batch, and returns the same result as a small batch."""
+    import torch
+    pop = _mix(8000, 43)
+    d, t0, t1 = 20.0, 0.0, 3999.0
+    ref = cds.screen(pop, t0, t1, 1.0, d, batch_object_steps=8000)
+    free, total = torch.cuda.mem_get_info()
+    hog = torch.empty(max(0, free - (6 << 30)), dtype=torch.uint8, device="cuda")   # leave ~6 GB
+    try:
+        got, st = cds.screen(pop, t0, t1, 1.0, d, batch_object_steps=10 ** 12, return_stats=True)
+    finally:
+        del hog
+        torch.cuda.empty_cache()
+    assert 1 <= st["grids_in_flight"] < 4000, st["grids_in_flight"]
+    assert np.array_equal(got, ref)
