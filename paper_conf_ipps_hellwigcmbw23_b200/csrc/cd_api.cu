@@ -748,7 +748,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     R.cand.st = st;
     if (ke <= kb || n < 2) return CD_OK;
 
-    const uint64_t M = next_pow2((uint64_t)std::max<int64_t>(2 * n, 64));   // >= 2n slots (power of 2)
+    const uint64_t M = next_pow2((uint64_t)std::max<int64_t>(2 * n, 256));   // >= 2n slots (power of 2, >= 256: one CSR allocation block per step)
     const uint64_t mask = M - 1;
     const size_t target = o.batch_object_steps ? o.batch_object_steps : (size_t(1) << 20);
     int64_t Bmax = std::max<int64_t>(1, (int64_t)(target / (size_t)n));

@@ -624,18 +624,30 @@ __global__ void k_csr_alloc(const Slot* __restrict__ slots, uint32_t* __restrict
         const unsigned long long w1 = slots[(size_t)s * M + h].head;
         cnt = (uint32_t)(w1 >> 32) == tag ? (uint32_t)w1 : 0u;
     }
-    // warp inclusive prefix sum (the warp's slots all belong to one step: M is a multiple of 32)
-    const unsigned lane = threadIdx.x & 31;
+    // block prefix sum (the block's 256 slots all belong to one step: M is a multiple of 256),
+    // one atomic per block on the step's total (one per warp serialised on the single counter)
+    __shared__ uint32_t s_w[8];
+    __shared__ unsigned long long s_base;
+    const unsigned lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     uint32_t inc = cnt;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
         const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
         if (lane >= (unsigned)o) inc += y;
     }
-    unsigned long long base = 0;
-    if (lane == 31 && in && inc) base = atomicAdd(total + s, (unsigned long long)inc);
-    base = __shfl_sync(0xffffffffu, base, 31);
-    if (in) start[(size_t)s * M + h] = (uint32_t)base + inc - cnt;
+    if (lane == 31) s_w[wid] = inc;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t run = 0;
+        for (int w = 0; w < 8; ++w) {
+            const uint32_t x = s_w[w];
+            s_w[w] = run;
+            run += x;
+        }
+        s_base = (in && run) ? atomicAdd(total + s, (unsigned long long)run) : 0ull;
+    }
+    __syncthreads();
+    if (in) start[(size_t)s * M + h] = (uint32_t)s_base + s_w[wid] + inc - cnt;
 }
 
 __global__ void k_csr_scatter(const Entry* __restrict__ tmp, const Slot* __restrict__ slots,
