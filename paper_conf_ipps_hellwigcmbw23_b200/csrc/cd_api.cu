@@ -765,8 +765,12 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     // can follow the cell edge chosen after the first round.  3 = CSR grid (sort + segment: the
     // open-addressing slots count each cell's objects, a counting sort makes each cell's entries
     // one contiguous segment).
-    const bool csr = o.grid_table == 3;
-    const bool can_chain = o.grid_table != 1 && !csr, can_open = o.grid_table != 2;
+    // sort + segment pays where the half-shell grid's cells are crowded: measured crossover (hybrid,
+    // 1M ... 8M objects at 9 s) at ~2.6 candidates per object-step -- 1M (1.4): open map 421 vs
+    // 459 us, 2M (2.6): even, 3M (3.9): -10 %, 4M (5.2): -25 %, 8M (10.4): -27 % per step
+    constexpr double kCsrDensity = 3.0;   // candidates per object-step from which grid_table 0 uses it
+    bool csr = o.grid_table == 3;
+    const bool can_chain = o.grid_table != 1 && o.grid_table != 3, can_open = o.grid_table != 2;
 #ifndef CD_CHAIN_FACTOR
 #define CD_CHAIN_FACTOR 8
 #endif
@@ -822,11 +826,14 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     DBuf<Entry> csr_tmp(st);
     DBuf<uint32_t> csr_start(st);
     DBuf<unsigned long long> csr_total(st);
-    if (csr) {
+    auto csr_alloc = [&]() -> cd_status {
+        if (csr_tmp.p) return CD_OK;
         CU(csr_tmp.alloc((size_t)Bmax * n));
         CU(csr_start.alloc(2 * (size_t)Bmax * M));
         CU(csr_total.alloc((size_t)Bmax));
-    }
+        return CD_OK;
+    };
+    if (csr) TRY(csr_alloc());
     static const bool no_pdl = getenv("CD_NO_PDL") != nullptr;   // A/B switch for experiments
     auto tab_of = [&](uint64_t b) {
         return GridTab{slotset[b % 2], bitset[b % 3],
@@ -928,6 +935,17 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                                     ? std::max<int64_t>(16, (int64_t)std::llround(64.0 / dt)) : 0;
     const int64_t resort_R = rs_opt < 0 ? 0 : rs_opt > 0 ? rs_opt : resort_auto;
     const bool spatial = resort_R > 0 && n >= 4096 && !csr;   // (CSR segments are cell-ordered)
+    // auto sort + segment (grid_table 0, half-shell map, no spatial order): from the a-priori
+    // density now, from the measured one once the first round has settled the cell edge
+    auto pick_csr = [&](double per_object_step) {
+        return o.grid_table == 3 ||
+               (o.grid_table == 0 && !spatial && g.halfshell && per_object_step >= kCsrDensity);
+    };
+    csr = pick_csr(est_step / std::max<double>(1.0, (double)n));
+    if (csr) {
+        chained = false;
+        TRY(csr_alloc());
+    }
     const int ncolH = S.j2 ? kNCol : kDOm;
     DBuf<double> Hrec[2] = {DBuf<double>(st), DBuf<double>(st)};
     DBuf<uint8_t> Hcls[2] = {DBuf<uint8_t>(st), DBuf<uint8_t>(st)};
@@ -1202,6 +1220,11 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
             g.halfshell = L < 2.0 * gc ? 1 : 0;
             const bool was_chained = chained;
             chained = pick_chained(g);
+            csr = pick_csr(dens);
+            if (csr) {
+                chained = false;
+                TRY(csr_alloc());
+            }
             if (chained != was_chained) {
                 // the bitmap / head sets change meaning (occupancy bits <-> epoch-tagged list
                 // heads): clear all three, stream-ordered after the round already in flight

@@ -120,3 +120,21 @@ def test_hybrid_counter_rotating_wide_windows():
     pop = popgen.counter_rotating(600, 7)
     res, st = _check(pop, 0.0, 3600.0, 9.0, 5.0)
     assert res["matched"] > 50
+
+
+def test_hybrid_crowded_cells_pick_sort_segment():
+    """grid_table 0 switches the half-shell grid to sort + segment when the measured coarse
+    candidate rate reaches 3 per object-step (crowded cells, e.g. 8M objects at 9 s): a dense
+    thin shell triggers it; the result equals the oracle and the forced open-addressing map."""
+    rng = np.random.default_rng(9)
+    n = 3000   # a 30 km thick, 1 rad long, +-0.05 rad wide swarm: ~5 coarse candidates per object
+    pop = {"a": rng.uniform(7000, 7030, n), "e": rng.uniform(0, 0.001, n),
+           "inc": 0.9 + rng.uniform(-0.05, 0.05, n), "raan": 0.3 + rng.uniform(-0.05, 0.05, n),
+           "argp": np.zeros(n), "nu0": rng.uniform(0, 1.0, n)}
+    res, st = _check(pop, 0.0, 900.0, 9.0, 2.0)
+    assert st["candidates"] / (st["steps"] * n) >= 3.0, st["candidates"] / (st["steps"] * n)
+    assert st["grid_table"] == 3
+    assert res["matched"] > 10
+    forced = cds.screen(pop, 0.0, 900.0, 9.0, 2.0, mode="hybrid", grid_table=1)
+    auto = cds.screen(pop, 0.0, 900.0, 9.0, 2.0, mode="hybrid")
+    assert np.array_equal(auto, forced)
