@@ -90,3 +90,33 @@ def test_bench_distributed_path_under_torchrun():
     assert line["merge"]["records_last_step"] > 0
     assert line["value"] > 0 and line["e2e"]["value"] > 0 and line["e2e"]["d2h_bytes_per_step"] > 0
     assert line["config"]["conjunctions"] > 0
+
+
+def test_nccl_merge_of_shards_times_slices():
+    """The two sharding axes (SURVEY 8(e) time slices x 8(f) radial object-space shards) through
+    the NCCL merge: 3 radial shards x 2 time slices screened on the device (shard members only,
+    R21), ids mapped to the caller's, gathered and sorted over the process group -- identical to
+    the whole screen, without duplicates."""
+    import torch
+    import torch.distributed as dist
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{_port()}", rank=0, world_size=1,
+                            device_id=torch.device("cuda", 0))
+    try:
+        pop = popgen.random_population(30000, 92, "catalog", 6000)
+        t0, t1, dt, d = 500.0, 1099.0, 1.0, 5.0
+        whole = cds.screen(pop, t0, t1, dt, d)
+        bounds = cdist.shell_bounds(pop, 3)
+        parts = []
+        for s in range(len(bounds) - 1):
+            for q in range(2):
+                r, _ = cdist.screen_shard(pop, t0, t1, dt, d, bounds, s, rank=q, n_ranks=2)
+                parts.append(torch.from_numpy(np.frombuffer(r.tobytes(), dtype=np.uint8).reshape(-1, 32).copy()))
+        local = torch.cat(parts[::-1]).cuda()
+        merged = cdist.merge_conjunctions(local, stream=torch.cuda.current_stream().cuda_stream)
+        torch.cuda.synchronize()
+        assert cdist.count_duplicates(merged) == 0
+        assert len(whole) > 50
+        assert np.array_equal(cdist.records_to_numpy(merged), whole)
+    finally:
+        dist.destroy_process_group()
