@@ -286,7 +286,7 @@ typedef struct {
     double capacity;                /* c = max(c', 10^4) * 2 * 2                             */
     double capacity_bytes;          /* g_ch = c * 16 B                                       */
     double fixed_bytes;             /* a_s + a_k + a_ch of this library: elements (48 B/object),
-                                       orbit records (325 B/object), first-round candidate queue
+                                       orbit records (85 B/object), first-round candidate queue
                                        (12 B/entry) and work items (24 B/entry)                      */
     double bytes_per_grid;          /* a_gh + a_l: one step's grid table + 32 B entries per object   */
     double grids_in_memory;         /* p = (m - a_s - a_k - a_ch) / (a_gh + a_l)             */

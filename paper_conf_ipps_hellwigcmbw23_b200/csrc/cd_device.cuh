@@ -24,14 +24,13 @@ enum Col : int {
     kAPx = 3, kAPy = 4, kAPz = 5,   // a * P (perifocal x axis)
     kBQx = 6, kBQy = 7, kBQz = 8,   // b * Q, b = a sqrt(1-e^2)
     kQper = 9,                       // perigee radius q = a(1-e) (acceleration bound)
-    kEcr = 10, kEsr = 11,            // e cos(rho), e sin(rho), rho = e/2   (real nodes)
-    kTab = 12,                       // 4 per symmetric interior pair: e cos(rho c_j),
-                                     // e sin(rho c_j), cosh(rho s_j), sinh(rho s_j)
+    // (the Contour constants of P:168 -- e cos(rho), e sin(rho) and the node tables -- are
+    // evaluated in registers by series, contour_core: no record columns)
     // J2 secular propagator (Orbits::j2): node and perigee rates and
     // the axis ratios that rotate the (aP, bQ) frame in its plane
-    kDOm = 40, kDw = 41,             // dOmega/dt, domega/dt [rad/s]
-    kBA = 42, kAB = 43,              // b/a, a/b
-    kNCol = 44
+    kDOm = 10, kDw = 11,             // dOmega/dt, domega/dt [rad/s]
+    kBA = 12, kAB = 13,              // b/a, a/b
+    kNCol = 14
 };
 
 // J2 secular propagator constants (EGM-96 / WGS-84, reading R19)
@@ -190,21 +189,51 @@ __constant__ double kNodes[5][7][4] = {
         {0.30901699437494745, 0.9510565162951535, -0.8090169943749473, 0.5877852522924732},
         {0.10452846326765346, 0.9945218953682733, -0.9781476007338057, 0.20791169081775931}}};
 
-// cos/sin and cosh/sinh of |x| <= 0.05 by 5-term Taylor polynomials (truncation < 3e-20):
-// the per-object Contour constants of eccentricity class 1 (rho = e/2 <= 0.05) are evaluated in
-// registers like class 0's instead of being streamed from the records (12 columns, 96 bytes per
-// object-step of the ~11 % class-1 objects of config 4)
-__device__ __forceinline__ void cs_series5(double x, double& c, double& s)
+// cos/sin and cosh/sinh of |x| <= rho_max(class) by T-term Taylor polynomials in Horner form
+// (T = 5 / 7 / 8 / 10 for rho <= 0.05 / 0.15 / 0.3 / 0.5: truncation < 3e-20 in every class, max
+// error vs libm 2.2e-16 absolute over each range): the per-object Contour constants
+// e cos(rho cos th_j), e sin(rho cos th_j), cosh(rho sin th_j), sinh(rho sin th_j) (P:168's
+// "precalculated reusable parts") are evaluated in registers instead of being streamed from the
+// records -- every class reads the same 9 columns per object-step (the tables were 80-240 bytes
+// per object-step of the ~16 % e > 0.01 objects; measured equal or faster in every class split)
+template <int T>
+__device__ __forceinline__ void cs_series(double x, double& c, double& s)
 {
     const double x2 = x * x;
-    c = fma(fma(fma(fma(1.0 / 40320.0, x2, -1.0 / 720.0), x2, 1.0 / 24.0), x2, -0.5), x2, 1.0);
-    s = x * fma(fma(fma(fma(1.0 / 362880.0, x2, -1.0 / 5040.0), x2, 1.0 / 120.0), x2, -1.0 / 6.0), x2, 1.0);
+    double pc = 0.0, ps = 0.0;
+#pragma unroll
+    for (int k = T - 1; k >= 0; --k) {   // x^{2k}: (-1)^k / (2k)!,  x^{2k+1}: (-1)^k / (2k+1)!
+        double f2k = 1.0;                // (compile-time constants once unrolled)
+#pragma unroll
+        for (int q = 2; q <= 2 * k; ++q) f2k *= (double)q;
+        const double f2k1 = f2k * (double)(2 * k + 1);
+        const double sg = (k & 1) ? -1.0 : 1.0;
+        pc = fma(pc, x2, sg / f2k);
+        ps = fma(ps, x2, sg / f2k1);
+    }
+    c = pc;
+    s = x * ps;
 }
-__device__ __forceinline__ void chsh_series5(double x, double& ch, double& sh)
+template <int T>
+__device__ __forceinline__ void chsh_series(double x, double& ch, double& sh)
 {
     const double x2 = x * x;
-    ch = fma(fma(fma(fma(1.0 / 40320.0, x2, 1.0 / 720.0), x2, 1.0 / 24.0), x2, 0.5), x2, 1.0);
-    sh = x * fma(fma(fma(fma(1.0 / 362880.0, x2, 1.0 / 5040.0), x2, 1.0 / 120.0), x2, 1.0 / 6.0), x2, 1.0);
+    double pc = 0.0, ps = 0.0;
+#pragma unroll
+    for (int k = T - 1; k >= 0; --k) {
+        double f2k = 1.0;
+#pragma unroll
+        for (int q = 2; q <= 2 * k; ++q) f2k *= (double)q;
+        const double f2k1 = f2k * (double)(2 * k + 1);
+        pc = fma(pc, x2, 1.0 / f2k);
+        ps = fma(ps, x2, 1.0 / f2k1);
+    }
+    ch = pc;
+    sh = x * ps;
+}
+__host__ __device__ constexpr int series_terms(int N)
+{
+    return N <= 6 ? 5 : N <= 8 ? 7 : N <= 12 ? 8 : 10;
 }
 
 template <int N>
@@ -224,14 +253,11 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
         const double x2 = rho * rho;
         ecr = e * fma(fma(fma(-1.0 / 720.0, x2, 1.0 / 24.0), x2, -0.5), x2, 1.0);
         esr = e * rho * fma(fma(fma(-1.0 / 5040.0, x2, 1.0 / 120.0), x2, -1.0 / 6.0), x2, 1.0);
-    } else if (N == 6) {   // class 1 (e <= 0.1): rho <= 0.05
+    } else {   // classes 1-4 (rho <= 0.05 / 0.15 / 0.3 / 0.5)
         double cr, sr;
-        cs_series5(rho, cr, sr);
+        cs_series<series_terms(N)>(rho, cr, sr);
         ecr = e * cr;
         esr = e * sr;
-    } else {
-        ecr = O.at(kEcr, r);
-        esr = O.at(kEsr, r);
     }
     // real nodes th = 0 (z = c + rho) and th = pi (z = c - rho)
     const double f0 = (dc + rho) - (sc * ecr + cc * esr);
@@ -259,17 +285,12 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
                 es = e * a * fma(fma(fma(-1.0 / 5040.0, a2, 1.0 / 120.0), a2, -1.0 / 6.0), a2, 1.0);
                 ch = fma(fma(fma(1.0 / 720.0, b2, 1.0 / 24.0), b2, 0.5), b2, 1.0);
                 sh = b * fma(fma(fma(1.0 / 5040.0, b2, 1.0 / 120.0), b2, 1.0 / 6.0), b2, 1.0);
-            } else if (N == 6) {   // class 1: arguments rho cos th, rho sin th <= 0.05
+            } else {   // arguments rho cos th, rho sin th <= rho
                 double cx, sx;
-                cs_series5(rho * ct, cx, sx);
+                cs_series<series_terms(N)>(rho * ct, cx, sx);
                 ec = e * cx;
                 es = e * sx;
-                chsh_series5(rho * st, ch, sh);
-            } else {
-                ec = O.at(kTab + 4 * (j - 1) + 0, r);
-                es = O.at(kTab + 4 * (j - 1) + 1, r);
-                ch = O.at(kTab + 4 * (j - 1) + 2, r);
-                sh = O.at(kTab + 4 * (j - 1) + 3, r);
+                chsh_series<series_terms(N)>(rho * st, ch, sh);
             }
             // point j (cos th = +ct) and its mirror N-1-j (cos th = -ct, same sin th)
             const double esin_a = sc * ec + cc * es, ecos_a = cc * ec - sc * es;

@@ -122,18 +122,7 @@ __global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, 
     put(kAPx, a * P[0]); put(kAPy, a * P[1]); put(kAPz, a * P[2]);
     put(kBQx, b * Q[0]); put(kBQy, b * Q[1]); put(kBQz, b * Q[2]);
     put(kQper, a * (1.0 - e));
-    const double rho = 0.5 * e;
-    put(kEcr, e * cos(rho));
-    put(kEsr, e * sin(rho));
     const int cl = max(ecc_class(e), min_cls);
-    const int N = class_points(cl);
-    for (int j = 1; j <= (N - 2) / 2; ++j) {
-        const double ct = kNodes[cl][j - 1][0], st = kNodes[cl][j - 1][1];
-        put(kTab + 4 * (j - 1) + 0, e * cos(rho * ct));
-        put(kTab + 4 * (j - 1) + 1, e * sin(rho * ct));
-        put(kTab + 4 * (j - 1) + 2, cosh(rho * st));
-        put(kTab + 4 * (j - 1) + 3, sinh(rho * st));
-    }
     cls[r] = (uint8_t)cl;
 }
 

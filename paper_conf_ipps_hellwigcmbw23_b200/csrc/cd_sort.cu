@@ -156,9 +156,8 @@ __global__ void k_space_keys(const Entry* __restrict__ E, const uint8_t* __restr
     val[t] = (uint32_t)t;
 }
 
-// new slot u takes old slot t = perm[u]: its build-record columns (classes 0 and 1: the 9 lean
-// columns plus the J2 rates -- their Contour constants are evaluated in registers; other classes:
-// all), class byte and internal id
+// new slot u takes old slot t = perm[u]: its build-record columns (the 9 that the build reads,
+// plus the J2 rates), class byte and internal id
 __global__ void k_resort_gather(const double* __restrict__ Hold, const uint8_t* __restrict__ cold,
                                 const uint32_t* __restrict__ sold, const uint32_t* __restrict__ perm,
                                 int64_t n, int ncol, int j2, double* __restrict__ Hnew,
@@ -167,12 +166,10 @@ __global__ void k_resort_gather(const double* __restrict__ Hold, const uint8_t* 
     const int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (u >= n) return;
     const uint32_t t = perm[u];
-    const uint8_t c = cold[t];
-    cnew[u] = c;
+    cnew[u] = cold[t];
     snew[u] = sold ? sold[t] : t;
-    const int lean = kBQz + 1;
-    for (int k = 0; k < (c <= 1 ? lean : ncol); ++k) Hnew[k * n + u] = Hold[k * n + t];
-    if (c <= 1 && j2)
+    for (int k = 0; k <= kBQz; ++k) Hnew[k * n + u] = Hold[k * n + t];
+    if (j2)
         for (int k = kDOm; k < ncol; ++k) Hnew[k * n + u] = Hold[k * n + t];
 }
 
