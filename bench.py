@@ -199,9 +199,16 @@ def run_ours(args):
     # timing) runs whenever there are several ranks, and also at one rank with --dist (torchrun
     # --nproc-per-node 1), so a one-GPU box exercises the same code path
     distributed = world > 1 or args.dist
+    # CD_BENCH_BACKEND=gloo (testing only): several ranks sharing one GPU, to exercise the
+    # multi-rank logic of this file on a one-GPU box; the product path is NCCL, one rank per GPU
+    backend = os.environ.get("CD_BENCH_BACKEND", "nccl")
     if distributed:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        gpu = local if backend == "nccl" else local % max(1, torch.cuda.device_count())
+        torch.cuda.set_device(gpu)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", gpu))
+        else:
+            dist.init_process_group(backend)
     else:
         torch.cuda.set_device(0)
     dev = torch.device("cuda", torch.cuda.current_device())
@@ -347,19 +354,24 @@ def run_ours(args):
                 hms.append(e0.elapsed_time(e1))
                 hst.append(st.as_dict())
         htot = float(np.sum(hms))
+        keys = ("candidates", "conjunctions", "hybrid_ap_rejected", "hybrid_coplanar",
+                "hybrid_path_rejected", "hybrid_time_rejected", "refined", "steps")
+        hsum = {k: int(sum(h[k] for h in hst)) for k in keys}
         if distributed:
             t = torch.tensor([htot], dtype=torch.float64, device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             htot = float(t.item())
-        hunits = float(n) * sum(h["steps"] for h in hst) * world
+            c = torch.tensor([hsum[k] for k in keys], dtype=torch.int64, device=dev)
+            dist.all_reduce(c)   # every rank's slices: the whole window
+            hsum = dict(zip(keys, (int(x) for x in c.tolist())))
+        hunits = float(n) * hsum["steps"]
         hyb = {"variant": "hybrid", "dt_s": cfg.dt_hybrid, "steps_in_window": Kh,
                "value": hunits / (htot / 1e3), "unit": "object-steps/s (coarse steps)",
                "wall_s_window": htot / 1e3,
-               "coarse_candidates": int(sum(h["candidates"] for h in hst)),
-               "conjunctions": int(sum(h["conjunctions"] for h in hst)),
-               "filter": {k: int(sum(h[k] for h in hst)) for k in
-                          ("hybrid_ap_rejected", "hybrid_coplanar", "hybrid_path_rejected",
-                           "hybrid_time_rejected", "refined")}}
+               "coarse_candidates": hsum["candidates"], "conjunctions": hsum["conjunctions"],
+               "filter": {k: hsum[k] for k in ("hybrid_ap_rejected", "hybrid_coplanar",
+                                               "hybrid_path_rejected", "hybrid_time_rejected",
+                                               "refined")}}
 
     # end to end through the public API with HOST buffers: pinned host inputs (H2D inside the
     # call), results back in host memory.  One rank: cd_screen with host results.  Distributed:

@@ -120,3 +120,25 @@ def test_nccl_merge_of_shards_times_slices():
         assert np.array_equal(cdist.records_to_numpy(merged), whole)
     finally:
         dist.destroy_process_group()
+
+
+def test_bench_two_ranks_share_one_gpu():
+    """bench.py's multi-rank logic (slices per rank, max-over-ranks time, summed units and counts,
+    the per-step merge, the e2e leg with the merge) at world size 2 on the one-GPU box, through
+    the gloo backend (CD_BENCH_BACKEND, testing only; the product path is NCCL, one rank per
+    GPU): the day's conjunctions over both ranks equal the stored oracle count of config 2."""
+    import json as _json
+    z = np.load(ROOT / "tests" / "golden" / "fullwindow_cfg2_grid.npz")
+    want = _json.loads(str(z["meta"]))["conjunctions"]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--standalone", "--nnodes=1",
+           "--nproc-per-node=2", str(ROOT / "bench.py"), "--config", "2", "--steps", "4",
+           "--warmup", "3", "--no-cpu-baseline", "--e2e-steps", "2"]
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1", CD_BENCH_BACKEND="gloo")
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    line = json.loads([x for x in r.stdout.splitlines() if x.startswith("{")][-1])
+    assert line["n_gpus"] == 2 and line["config"]["slices"] == 8
+    assert line["config"]["conjunctions"] == want
+    assert line["merge"]["ranks"] == 2 and line["merge"]["duplicates_last_step"] == 0
+    assert line["hybrid"]["steps_in_window"] == 9601
+    assert line["e2e"]["value"] > 0
