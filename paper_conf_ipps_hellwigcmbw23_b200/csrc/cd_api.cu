@@ -926,8 +926,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     // slots; every R steps the slots are renumbered in Morton order of the positions of the last
     // built step.  Hot build records / class bytes / slot -> internal id map, double-buffered:
     // a launch builds batch b + 1 in the new order while it scans batch b in the old one.
-    static const char* env_rs = getenv("CD_RESORT_STEPS");   // A/B switch for experiments
-    const int rs_opt = env_rs ? atoi(env_rs) : o.resort_steps;
+    const int rs_opt = o.resort_steps;
     // auto: on for populations whose per-step grid is far beyond L2 (>= 4M objects, grid variant;
     // measured at 8M: 894 -> 785 us per step with R = 64 at dt = 1 s), off below (at 1M the
     // re-sort costs more than the locality returns: 60.3 vs 61.4 us per step)
