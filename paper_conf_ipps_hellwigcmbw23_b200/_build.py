@@ -30,14 +30,30 @@ def up_to_date() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False) -> Path:
+    """Compile every translation unit in parallel (nvcc, sm_100a), then link the shared
+    library (no device code crosses translation units, so no relocatable device code)."""
     if not force and up_to_date():
         return LIB
+    import tempfile
     nvcc = os.environ.get("NVCC", "nvcc")
+    compile_flags = [f for f in NVCC_FLAGS if f != "-shared"]
     tmp = LIB.with_suffix(f".so.tmp{os.getpid()}")
-    cmd = [nvcc] + NVCC_FLAGS + ["-o", str(tmp)] + [str(s) for s in sources()]
-    if verbose:
-        print(" ".join(cmd))
-    subprocess.run(cmd, check=True)
+    with tempfile.TemporaryDirectory(prefix="cdbuild") as td:
+        objs, procs = [], []
+        for src in sources():
+            obj = Path(td) / (src.stem + ".o")
+            cmd = [nvcc] + compile_flags + ["-c", "-o", str(obj), str(src)]
+            if verbose:
+                print(" ".join(cmd))
+            procs.append((cmd, subprocess.Popen(cmd)))
+            objs.append(str(obj))
+        for cmd, p in procs:
+            if p.wait() != 0:
+                raise subprocess.CalledProcessError(p.returncode, cmd)
+        link = [nvcc, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", str(tmp)] + objs
+        if verbose:
+            print(" ".join(link))
+        subprocess.run(link, check=True)
     os.replace(tmp, LIB)
     return LIB
 
