@@ -65,3 +65,56 @@ def test_random_options_match_oracle(seed):
     Co = oracle.conjunctions(pop, t0, t1, dt, d, gc, Ko)
     res = parity.compare_conjunctions(pop, Cg, Co, t0, t1, dt, d, gc)
     assert res["one_sided"] == 0, (kw, res)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_random_options_hybrid_match_oracle(seed):
+    rng = np.random.default_rng(6000 + seed)
+    n = int(rng.integers(1000, 8000))
+    pop = popgen.random_population(n, 7000 + seed, "catalog", int(rng.integers(0, n // 2)))
+    d = float(rng.choice([2.0, 5.0, 10.0]))
+    dt = float(rng.choice([3.0, 9.0, 15.0]))
+    t0 = float(rng.uniform(0, 5000))
+    t1 = t0 + dt * int(rng.integers(10, 60))
+    kw = _options(rng)
+    kw.pop("kepler_points", None)
+    gc = oracle.cell_size(d, dt)
+    Cg, st = cds.screen(pop, t0, t1, dt, d, mode="hybrid", return_stats=True, **kw)
+    Co, cnt = oracle.hybrid(pop, t0, t1, dt, d)
+    res = parity.compare_conjunctions(pop, Cg, Co, t0, t1, dt, d, gc)
+    assert res["one_sided"] == 0, (kw, res)
+    assert st["candidates"] == cnt["candidates"]
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_j2_and_legacy_match_oracle(seed):
+    rng = np.random.default_rng(8000 + seed)
+    n = int(rng.integers(300, 1500))
+    pop = popgen.random_population(n, 9000 + seed, "catalog", int(rng.integers(0, n // 3)))
+    d = float(rng.choice([10.0, 30.0]))
+    t0, dt = float(rng.uniform(0, 3000)), 1.0
+    t1 = t0 + int(rng.integers(20, 60))
+    gc = oracle.cell_size(d, dt)
+    kw = _options(rng)
+    kw.pop("kepler_points", None)
+    pj = dict(pop, propagator="j2")
+    Kg = cds.candidates(pj, t0, t1, dt, d, **kw)
+    Ko = oracle.candidates_grid(pj, t0, t1, dt, gc)
+    parity.compare_candidates(pj, Kg, Ko, t0, dt, gc)
+    Cg = cds.screen(pj, t0, t1, dt, d, **kw)
+    Co = oracle.conjunctions(pj, t0, t1, dt, d, gc, Ko)
+    assert parity.compare_conjunctions(pj, Cg, Co, t0, t1, dt, d, gc)["one_sided"] == 0
+    # legacy chain on a dense swarm (its pairs split over two ranks for odd seeds)
+    m = 800
+    pop = {"a": rng.uniform(7000, 7010, m), "e": rng.uniform(0, 0.001, m),
+           "inc": 0.9 + rng.uniform(-0.05, 0.05, m), "raan": 0.3 + rng.uniform(-0.05, 0.05, m),
+           "argp": np.zeros(m), "nu0": rng.uniform(0, 0.5, m)}
+    t1 = t0 + 300.0
+    Lg = cds.screen(pop, t0, t1, dt, d, mode="legacy", rank=seed % 2, n_ranks=1 + seed % 2)
+    Lo, _ = oracle.legacy(pop, t0, t1, dt, d)
+    if seed % 2:
+        Lg2 = cds.screen(pop, t0, t1, dt, d, mode="legacy", rank=0, n_ranks=2)
+        Lg = np.concatenate([Lg2, Lg])
+        Lg = Lg[np.lexsort((Lg["step"], Lg["j"], Lg["i"]))]
+    assert len(Lo) > 5
+    parity.compare_legacy(pop, Lg, Lo, t0, t1, dt, d)
