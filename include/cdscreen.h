@@ -161,6 +161,11 @@ typedef struct {
                                   test); with cell_factor = 1 and grid_table = 1 this is the
                                   paper's count of object pairs in the same or neighbouring cells
                                   (each unordered pair once per step)                */
+    uint64_t digest;           /* digest_only: sum mod 2^64 over the conjunctions of
+                                  i * 0x9E3779B1 + j * 0x85EBCA77 + step * 0xC2B2AE3D (caller ids,
+                                  i < j): order-independent, additive over time slices and ranks */
+    uint64_t digest_conjunctions; /* digest_only: the number of conjunctions digested          */
+    double min_pca;            /* digest_only: the smallest PCA [km] (+inf if none)            */
 } cd_stats;
 
 typedef struct {
@@ -232,6 +237,12 @@ typedef struct {
     int emit_raw_counts;      /* also count the pairs the scan examines into cd_stats.raw_pairs
                                  (the paper's raw count with cell_factor = 1, grid_table = 1;
                                  P:95); default 0                                   */
+    int digest_only;          /* 1: do not return the conjunctions -- fold each round's records
+                                 into cd_stats.digest / digest_conjunctions / min_pca on the
+                                 device and reuse the buffer (for screens whose result does not
+                                 fit memory, e.g. 8M objects x 7 days: ~4e9 records);
+                                 the result is {NULL, 0}.  CD_GRID / CD_HYBRID without in-library
+                                 shards; default 0                                               */
 } cd_options;
 
 /* Fill *opt with the defaults above. */

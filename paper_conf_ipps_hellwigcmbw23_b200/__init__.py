@@ -76,7 +76,8 @@ class cd_stats(C.Structure):
                 ("launches_propagate", C.c_uint64), ("launches_insert", C.c_uint64),
                 ("launches_scan", C.c_uint64), ("launches_refine", C.c_uint64),
                 ("step_launches", C.c_uint64), ("cell_factor", C.c_double), ("grid_table", C.c_int),
-                ("grids_in_flight", C.c_uint64), ("raw_pairs", C.c_uint64)]
+                ("grids_in_flight", C.c_uint64), ("raw_pairs", C.c_uint64), ("digest", C.c_uint64),
+                ("digest_conjunctions", C.c_uint64), ("min_pca", C.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -96,7 +97,8 @@ class cd_options(C.Structure):
                 ("stats", C.POINTER(cd_stats)), ("propagator", C.c_int),
                 ("shell_lo", C.c_double), ("shell_hi", C.c_double),
                 ("alloc", ALLOC_FN), ("free", FREE_FN), ("alloc_ctx", C.c_void_p),
-                ("shards", C.c_int), ("resort_steps", C.c_int), ("emit_raw_counts", C.c_int)]
+                ("shards", C.c_int), ("resort_steps", C.c_int), ("emit_raw_counts", C.c_int),
+                ("digest_only", C.c_int)]
 
 
 class cd_plan_info(C.Structure):
@@ -315,7 +317,8 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
                  cell_factor=None, batch_object_steps=None, round_steps=None,
                  outputs_on_device=False, inputs_on_device=False, profile_phases=False,
                  l2_persist=None, grid_table=None, propagator=None, shell=None, allocator=None,
-                 shards=None, kepler_points=None, resort_steps=None, emit_raw_counts=False):
+                 shards=None, kepler_points=None, resort_steps=None, emit_raw_counts=False,
+                 digest_only=False):
     o = cd_options()
     cd_options_init(o)
     o.rank, o.n_ranks = rank, n_ranks
@@ -361,6 +364,7 @@ def make_options(rank=0, n_ranks=1, v_margin=None, grid_origin=None, device=None
     if resort_steps is not None:
         o.resort_steps = int(resort_steps)
     o.emit_raw_counts = int(bool(emit_raw_counts))
+    o.digest_only = int(bool(digest_only))
     return o
 
 
@@ -479,6 +483,16 @@ def propagate(pop, times, velocity=False, **kw):
                         v.ctypes.data if velocity else None, opt))
     return (xyz, v) if velocity else xyz
 
+
+
+def conjunction_digest(conj):
+    """The digest of a conjunction array as cd_stats.digest defines it (cdscreen.h): sum mod 2^64
+    of i * 0x9E3779B1 + j * 0x85EBCA77 + step * 0xC2B2AE3D."""
+    if len(conj) == 0:
+        return 0
+    h = (conj["i"].astype(np.uint64) * np.uint64(0x9E3779B1) + conj["j"].astype(np.uint64) * np.uint64(0x85EBCA77)
+         + conj["step"].astype(np.uint64) * np.uint64(0xC2B2AE3D))
+    return int(np.sum(h, dtype=np.uint64))
 
 
 def release_caches(device=-1):

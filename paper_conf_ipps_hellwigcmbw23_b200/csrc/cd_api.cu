@@ -720,6 +720,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
     stats.steps = (uint64_t)(ke - kb);
     stats.object_steps = (uint64_t)(ke - kb) * (uint64_t)n;
     const double gc = d + o.v_margin * dt;   // Eq. 1
+    const bool digest = o.digest_only && want == Want::Conj;
     // grid cell edge L = m g_c (m = cell_factor; 0 = auto: start from the a-priori density, then
     // choose from the candidate density measured in the first round, see choose_cell_factor)
     const bool auto_cell = o.cell_factor == 0.0;
@@ -1086,6 +1087,8 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         }
         CU(cudaMemcpyAsync(hslot[slot], ctrl.p, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
         CU(cudaMemcpyAsync(hnw[slot], nwork.p, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+        if (digest)   // after the snapshot: the snapshot's digest is that of the rounds before
+            CU(launch_conj_digest(R.conj.p, ocap, S.perm.p, ctrl.p, st, C.lc));
         CU(cudaEventRecord(rev[slot], st));
         DBG("round: enqueued", (long long)kr, (long long)Rk);
         return CD_OK;
@@ -1185,7 +1188,7 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
                                cudaMemcpyDeviceToDevice, st));
             R.n_cand += hctrl->n_cand;
         }
-        conj_before = hctrl->n_conj;
+        conj_before = digest ? 0 : hctrl->n_conj;   // (digest_only: the buffer was emptied)
         hyb_before[0] = hctrl->n_ap;
         hyb_before[1] = hctrl->n_coplanar;
         hyb_before[2] = hctrl->n_path;
@@ -1245,6 +1248,18 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         }
     }
     R.n_conj = (size_t)conj_before;
+    if (digest) {   // the last round's digest ran after its snapshot: read the final counters
+        Ctrl fin;
+        CU(cudaMemcpyAsync(&fin, ctrl.p, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
+        CU(cudaStreamSynchronize(st));
+        stats.digest = fin.dg_sum;
+        stats.digest_conjunctions = fin.dg_count;
+        const unsigned long long bits = ~fin.dg_notminpca;
+        double mp;
+        memcpy(&mp, &bits, sizeof mp);
+        stats.min_pca = fin.dg_count ? mp : INFINITY;
+        R.n_conj = 0;
+    }
     stats.cell_factor = L / gc;
     stats.grid_table = csr ? 3 : chained ? 2 : 1;
     stats.hybrid_ap_rejected = hyb_before[0];
@@ -1471,6 +1486,8 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
         return fail(CD_EINVAL, "CD_HYBRID and CD_LEGACY need CD_PROP_KEPLER (the filters assume fixed orbit planes)");
     if (mode == CD_LEGACY && o.shell_hi != 0.0)
         return fail(CD_EINVAL, "CD_LEGACY splits pairs by rank; radial shards apply to the grid");
+    if (o.digest_only && (mode == CD_LEGACY || o.shards > 1))
+        return fail(CD_EINVAL, "digest_only needs CD_GRID or CD_HYBRID without in-library shards");
     int64_t K = 0;
     TRY(validate_scalars(n, t0, t1, dt, d, o, &K));
     cd_stats stats;
@@ -1537,7 +1554,7 @@ cd_status screen_impl(const cd_elements* el, size_t n, double t0, double t1, dou
     float ms = 0.f;
     cudaEventElapsedTime(&ms, C.ev0, C.ev1);
     stats.ms_total = ms;
-    stats.conjunctions = R.n_conj;
+    stats.conjunctions = o.digest_only ? stats.digest_conjunctions : R.n_conj;
     stats.kernel_launches = C.lc.n;
     C.pt.harvest();
     C.pt.to_stats(stats);

@@ -633,6 +633,9 @@ struct Ctrl {   // device-side counters and flags of one call
     int err_range;
     int err_internal;
     unsigned long long n_raw;   // pairs examined by the scan (emit_raw_counts; per round)
+    // digest_only: accepted rounds' conjunctions folded into a count, an order-independent sum of
+    // hashes of (i, j, step) in caller ids, and the smallest PCA (stored as max of ~bits)
+    unsigned long long dg_count, dg_sum, dg_notminpca;
 };
 
 }  // namespace cdk

@@ -140,6 +140,11 @@ cudaError_t launch_brent(const cdk::Orbits& O, const RefineParams& p, const Work
                          const unsigned long long* n_work, size_t wcap, cdk::Conj* out,
                          size_t ocap, cdk::Ctrl* ctrl, cudaStream_t st, LaunchCount& lc);
 
+// digest_only: fold a round's records into Ctrl's digest and empty the buffer (k_conj_digest,
+// k_conj_reset; skipped for an overflowed round)
+cudaError_t launch_conj_digest(const cdk::Conj* c, size_t ocap, const uint32_t* perm, cdk::Ctrl* ctrl,
+                               cudaStream_t st, LaunchCount& lc);
+
 // ---- finalize (a10) --------------------------------------------------------------------
 // Map internal indices to external ids (i < j) and sort by (i, j, step).  Returns the sorted
 // array in `out` (device).  Scratch is allocated on the stream.

@@ -938,6 +938,51 @@ __global__ void __launch_bounds__(128) k_brent(Orbits O, RefineParams P, const W
     }
 }
 
+// digest_only (cd_options.digest_only): fold the round's conjunction records [0, n_conj) into the
+// digest (count, sum of hash(i, j, step) in caller ids, smallest PCA) unless the round overflowed
+// (n_conj > ocap: the host redoes it), then empty the buffer for the next round (k_conj_reset)
+__global__ void k_conj_digest(const Conj* __restrict__ c, size_t ocap, const uint32_t* __restrict__ perm,
+                              Ctrl* ctrl)
+{
+    const unsigned long long n = ctrl->n_conj;
+    if (n > ocap) return;
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    unsigned long long sum = 0, nmin = 0;
+    for (size_t k = blockIdx.x * (size_t)blockDim.x + threadIdx.x; k < n; k += stride) {
+        const Conj r = c[k];
+        uint32_t a = perm[r.i], b = perm[r.j];
+        if (a > b) { const uint32_t t = a; a = b; b = t; }
+        sum += (unsigned long long)a * 0x9E3779B1ull + (unsigned long long)b * 0x85EBCA77ull +
+               (unsigned long long)r.step * 0xC2B2AE3Dull;
+        const unsigned long long nb = ~(unsigned long long)__double_as_longlong(r.pca);
+        nmin = nb > nmin ? nb : nmin;
+    }
+    for (int o = 16; o; o >>= 1) {
+        sum += __shfl_down_sync(0xffffffffu, sum, o);
+        const unsigned long long y = __shfl_down_sync(0xffffffffu, nmin, o);
+        nmin = y > nmin ? y : nmin;
+    }
+    if ((threadIdx.x & 31) == 0) {
+        if (sum) atomicAdd(&ctrl->dg_sum, sum);
+        if (nmin) atomicMax(&ctrl->dg_notminpca, nmin);
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(&ctrl->dg_count, n);
+}
+
+__global__ void k_conj_reset(size_t ocap, Ctrl* ctrl)
+{
+    if (ctrl->n_conj <= ocap) ctrl->n_conj = 0;
+}
+
+cudaError_t launch_conj_digest(const Conj* c, size_t ocap, const uint32_t* perm, Ctrl* ctrl,
+                               cudaStream_t st, LaunchCount& lc)
+{
+    k_conj_digest<<<148 * 4, 256, 0, st>>>(c, ocap, perm, ctrl);
+    k_conj_reset<<<1, 1, 0, st>>>(ocap, ctrl);
+    lc.bump(2);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_prefilter(const Orbits& O, const RefineParams& p, const Cand* q, size_t qcap,
                              Work* w, size_t wcap, unsigned long long* n_work, Conj* out, size_t ocap,
                              Ctrl* ctrl, cudaStream_t st, LaunchCount& lc)

@@ -349,3 +349,26 @@ def test_memory_bounded_batch():
         torch.cuda.empty_cache()
     assert 1 <= st["grids_in_flight"] < 4000, st["grids_in_flight"]
     assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("mode,dt,kw", [("grid", 1.0, {}), ("grid", 1.0, dict(round_steps=3)),
+                                        ("hybrid", 9.0, {}), ("grid", 1.0, dict(resort_steps=2))])
+def test_digest_only_equals_full_result(mode, dt, kw):
+    """cd_options.digest_only: no records returned; the device-side digest (count, hash sum, min
+    PCA) equals the one computed from the full result, and is additive over time slices."""
+    pop = _mix(20000, 51, "catalog", 4000)
+    d, t0 = 10.0, 300.0
+    t1 = t0 + 120 * dt
+    full = cds.screen(pop, t0, t1, dt, d, mode=mode, **kw)
+    res, st = cds.screen(pop, t0, t1, dt, d, mode=mode, digest_only=True, return_stats=True, **kw)
+    assert len(res) == 0 and len(full) > 50
+    assert st["conjunctions"] == st["digest_conjunctions"] == len(full)
+    assert st["digest"] == cds.conjunction_digest(full)
+    assert st["min_pca"] == float(full["pca"].min())
+    tot, cnt = 0, 0
+    for q in range(3):
+        _, s2 = cds.screen(pop, t0, t1, dt, d, mode=mode, digest_only=True, rank=q, n_ranks=3,
+                           return_stats=True, **kw)
+        tot = (tot + s2["digest"]) % (1 << 64)
+        cnt += s2["digest_conjunctions"]
+    assert tot == st["digest"] and cnt == len(full)
