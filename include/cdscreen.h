@@ -195,9 +195,9 @@ typedef struct {
                                  2 = chained spatial hash (lists per hashed bucket, one atomic
                                  exchange per object); 3 = sort + segment (the open-addressing
                                  slots count each cell's objects, a counting sort by cell makes
-                                 each cell one contiguous segment); 0 = default (per geometry:
-                                 2 in ball mode; in half-shell mode 1, or 3 once the measured
-                                 candidate rate reaches 3 per object-step -- crowded cells).
+                                 each cell one contiguous segment); 0 = default (2; in
+                                 half-shell mode 3 once the measured candidate rate reaches 3
+                                 per object-step -- crowded cells).
                                  Results are identical; other values CD_EINVAL.                  */
     cd_stats* stats;          /* optional output                                              */
     int propagator;           /* cd_propagator; default CD_PROP_KEPLER                        */

@@ -512,6 +512,7 @@ __device__ __forceinline__ uint32_t bit_hash(int cx, int cy, int cz)
 #define CD_SB_BITS 2   // 4x4x4 superblocks (measured: 8M objects 970 -> 894 us per step, 1M 61.6 -> 60.3)
 #endif
 constexpr int kSB = CD_SB_BITS;
+static_assert(kSB >= 2, "the half-shell chained scan needs the 27 cells of a 3x3x3 block in distinct buckets");
 __device__ __forceinline__ uint32_t chain_bucket(int cx, int cy, int cz, uint32_t hmask)
 {
     constexpr uint32_t m = (1u << kSB) - 1u;

@@ -485,30 +485,11 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
 //    the own cell are walked; only entries tagged with the probed cell count (walk_bucket_tag),
 //    so a pair in cells A != B is reported once, by the object whose cell is lexicographically
 //    smaller (parity hashing keeps these buckets distinct from each other and the own bucket);
-//  * half-shell mode (L < 2 g_c, rare with this table): all 26 neighbour buckets, de-duplicated,
-//    are walked in full and a pair is reported only from its smaller id (walk_bucket_gt).
+//  * half-shell mode (L < 2 g_c): the buckets of the 13 half-shell neighbour cells, again only
+//    the probed cell's entries (needs 4x4x4 or larger superblocks, see below).
 __device__ __forceinline__ uint32_t head_index(uint32_t h, uint32_t epoch)
 {
     return ((h >> kEpochShift) == epoch && (h & kIdxMask)) ? (h & kIdxMask) - 1u : kNil;
-}
-
-// half-shell mode (26 neighbour buckets, each walked in full): report from the smaller id
-__device__ __forceinline__ void walk_bucket_gt(const GridGeom& g, const Entry* __restrict__ E,
-                                               uint32_t h, uint32_t epoch, uint32_t r, const double p[3],
-                                               uint32_t step, Cand* __restrict__ q, size_t qcap,
-                                               Ctrl* ctrl)
-{
-    uint32_t j = head_index(h, epoch);
-    uint32_t guard = g.max_walk;
-    while (j != kNil) {
-        if (guard-- == 0) {
-            ctrl->err_internal = 1;
-            return;
-        }
-        const Entry ej = E[j];
-        if (j > r) test_pair(g, r, j, p, ej, step, q, qcap, ctrl);
-        j = ej.next;
-    }
 }
 
 // ball mode: bucket of the probed cell (tag ctag), which lies in the positive half-space of the
@@ -548,20 +529,26 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
     if (!cell_of(g, p, c, fr)) return;
     // own bucket: successors only, every pair once (by the later-inserted object)
     walk(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
-    if (g.halfshell) {   // L < 2 g_c: all 26 neighbour cells (rare configuration; local arrays)
-        const uint32_t own = chain_bucket(c[0], c[1], c[2], hmask);
-        uint32_t bk[26];
-        int nb = 0;
-        for (int dx = -1; dx <= 1; ++dx)
-            for (int dy = -1; dy <= 1; ++dy)
-                for (int dz = -1; dz <= 1; ++dz) {
-                    const uint32_t b = chain_bucket(c[0] + dx, c[1] + dy, c[2] + dz, hmask);
-                    bool dup = b == own;
-                    for (int k = 0; k < nb; ++k) dup = dup || bk[k] == b;
-                    if (!dup) bk[nb++] = b;
-                }
-        for (int k = 0; k < nb; ++k)
-            walk_bucket_gt(g, E, __ldg(heads + bk[k]), epoch, (uint32_t)r, p, step, q, qcap, ctrl);
+    if (g.halfshell) {
+        // L < 2 g_c: the 13 half-shell neighbour cells (each unordered pair of cells of a 3x3x3
+        // block once, as in do_scan), only the probed cell's entries (tag).  The 27 cells of a
+        // 3x3x3 block differ pairwise in (c mod 4) on some axis, so with superblock buckets they
+        // never share a bucket: a colliding cell in the own bucket is never a neighbour (its
+        // entries fail the distance test), and no pair is seen from two buckets.
+        uint32_t hit = 0;
+#pragma unroll
+        for (int o = 1; o < 14; ++o) {
+            const uint32_t h = __ldg(heads + chain_bucket(c[0] + kHalfShell[o][0], c[1] + kHalfShell[o][1],
+                                                          c[2] + kHalfShell[o][2], hmask));
+            hit |= (head_index(h, epoch) != kNil ? 1u : 0u) << o;
+        }
+        while (hit) {
+            const int o = __ffs(hit) - 1;
+            hit &= hit - 1;
+            const int cx = c[0] + kHalfShell[o][0], cy = c[1] + kHalfShell[o][1], cz = c[2] + kHalfShell[o][2];
+            walk_bucket_tag(g, E, __ldg(heads + chain_bucket(cx, cy, cz, hmask)), epoch, cell_tag(cx, cy, cz),
+                            (uint32_t)r, p, step, q, qcap, ctrl);
+        }
         return;
     }
     const double rl = g.reach * g.inv_cell;

@@ -51,7 +51,7 @@ def test_hybrid_catalog_30k():
     assert res["matched"] > 30
 
 
-@pytest.mark.parametrize("table", [0, 3])
+@pytest.mark.parametrize("table", [0, 2, 3])
 def test_hybrid_shells_100k(table):
     pop, cfg, _ = popgen.make_config(3)
     res, st = _check(pop, 3600.0, 5400.0, 9.0, 2.0, grid_table=table)

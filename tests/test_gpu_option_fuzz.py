@@ -52,8 +52,6 @@ def test_random_options_match_oracle(seed):
     t0 = float(rng.uniform(0, 5000))
     t1 = t0 + dt * int(rng.integers(10, 80))
     kw = _options(rng)
-    if kw.get("grid_table") == 2 and kw.get("cell_factor", 4.0) < 2.0:
-        kw["grid_table"] = 0   # (chained + half-shell is valid but slow; keep the test short)
     gc = oracle.cell_size(d, dt)
     Kg = cds.candidates(pop, t0, t1, dt, d, **kw)
     Ko = oracle.candidates_grid(pop, t0, t1, dt, gc)
