@@ -493,6 +493,7 @@ __global__ void k_validate(Elements el, int64_t n, int* bad)
 // Device-resident orbit records of one call (internal order sorted by eccentricity class).
 struct OrbitSet {
     DBuf<double> rec;
+    DBuf<double> arec;     // refinement records (object-major, kAoS doubles per object)
     DBuf<uint8_t> cls;
     DBuf<uint32_t> perm;   // internal -> caller index
     int64_t n0 = 0;        // class-0 objects (sorted first)
@@ -501,6 +502,7 @@ struct OrbitSet {
     {
         Orbits O;
         O.rec = rec.p;
+        O.arec = arec.p;
         O.cls = cls.p;
         O.n = (int64_t)perm.n;
         O.n0 = n0;
@@ -514,7 +516,7 @@ cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_opti
     if (!el || !el->a || !el->e || !el->inc || !el->raan || !el->argp || !el->nu0)
         return fail(CD_EINVAL, "elements must be non-NULL");
     cudaStream_t st = C.st;
-    S.rec.st = S.cls.st = S.perm.st = st;
+    S.rec.st = S.arec.st = S.cls.st = S.perm.st = st;
     DBuf<double> up(st);
     Elements E;
     const double* src[6] = {el->a, el->e, el->inc, el->raan, el->argp, el->nu0};
@@ -555,8 +557,9 @@ cd_status prepare_orbits(Call& C, const cd_elements* el, size_t n, const cd_opti
     CU(sort_pairs_u32(key.p, keyo.p, idx.p, S.perm.p, n, 3, st, C.lc));
     S.j2 = o.propagator == CD_PROP_J2;
     CU(S.rec.alloc((size_t)(S.j2 ? kNCol : kDOm) * n));   // the J2 columns only when used
+    CU(S.arec.alloc((size_t)kAoS * n));
     CU(S.cls.alloc(n));
-    CU(launch_build_records(E, S.perm.p, (int64_t)n, S.rec.p, S.cls.p, S.j2, min_cls, st, C.lc));
+    CU(launch_build_records(E, S.perm.p, (int64_t)n, S.rec.p, S.arec.p, S.cls.p, S.j2, min_cls, st, C.lc));
     C.pt.stop();
     CU(cudaStreamSynchronize(st));   // hn0 is needed on the host
     S.n0 = (int64_t)hn0;
@@ -1207,7 +1210,10 @@ cd_status run(Call& C, const OrbitSet& S, double t0, double t1, double dt, doubl
         // so a long screen grows it early (little to copy) and rarely
         const double done_steps = (double)(rd.k + rd.Rk - kb);
         const double proj_conj = (double)conj_before * (double)(ke - kb) / std::max(1.0, done_steps);
-        if (want == Want::Conj && settled && (1.25 * proj_conj > (double)ocap || conj_before > ocap * 9 / 10)) {
+        // (from the first round on: it runs alone, so growing after it leaves no round in flight
+        // with the old capacity -- measured: a first growth one round later made the round then in
+        // flight overflow and be redone, 118 of 200 steps at 8M objects)
+        if (want == Want::Conj && (1.25 * proj_conj > (double)ocap || conj_before > ocap * 9 / 10)) {
             const size_t ncap = std::max<size_t>(2 * ocap, (size_t)(1.5 * proj_conj));
             DBG("grow: output", (long long)ocap, (long long)ncap);
             CU(R.conj.grow(ncap, ocap, st));
@@ -1785,11 +1791,11 @@ cd_status cd_plan(size_t n, double t0, double t1, double dt, double d, cd_mode m
         out->est_candidates_per_step = extra_p_candidates(nn, dt, dt, d, mode);
         out->capacity = std::max(out->est_candidates, 1e4) * 2.0 * 2.0;
         out->capacity_bytes = out->capacity * 16.0;
-        // this library's structures: a_s elements, a_k orbit records + class +
-        // permutation, a_ch the round's candidate queue (12 B) and work items (24 B)
+        // this library's structures: a_s elements, a_k orbit records (column- and
+        // object-major) + class + permutation, a_ch the round's candidate queue (12 B) and work items (24 B)
         const double qcap = (double)initial_qcap((int64_t)n, std::max(1.0, out->est_candidates_per_step));
         const double wcap = std::min(qcap, std::max(4194304.0, 4.0 * nn));
-        out->fixed_bytes = 48.0 * nn + (8.0 * kDOm + 1.0 + 4.0) * nn + 12.0 * qcap + 24.0 * wcap;
+        out->fixed_bytes = 48.0 * nn + (8.0 * kDOm + 8.0 * kAoS + 1.0 + 4.0) * nn + 12.0 * qcap + 24.0 * wcap;
         // a_gh + a_l of one step's grid, in the structure the auto cell edge selects for the
         // a-priori density: chained heads (4 B x next_pow2(8n)) in ball mode, the open map
         // (16 B x next_pow2(2n) slots + next_pow2(32n)-bit occupancy) in half-shell mode, plus the

@@ -53,8 +53,17 @@ __host__ __device__ inline int kepler_class_of_points(int pts)
     return pts == 0 || pts == 4 ? 0 : pts == 6 ? 1 : pts == 8 ? 2 : pts == 12 ? 3 : pts == 16 ? 4 : -1;
 }
 
+// Refinement records (Orbits::arec): the same columns object-major, one 128-byte line per object
+// (column c of object r at arec[r * kAoS + c], the class at kAoSCls): the refinement gathers a
+// candidate's two objects at random, and one line per object replaces up to 14 scattered sectors
+// of the column-major records (8M objects: the prefilter was DRAM-bound on those gathers).
+constexpr int kAoS = 16;
+constexpr int kAoSCls = 14;
+static_assert(kNCol <= kAoSCls, "refinement record columns");
+
 struct Orbits {
     const double* rec;   // kNCol x n
+    const double* arec;  // refinement records, n x kAoS (object-major)
     const uint8_t* cls;  // eccentricity class per object
     int64_t n;
     int64_t n0;          // objects [0, n0) are class 0 (records sorted by class)
@@ -62,6 +71,10 @@ struct Orbits {
     // records are streamed once per step: evict-first so they do not push the per-step grid
     // (slots, bitmap, entries) out of L2
     __device__ __forceinline__ double at(int c, int64_t r) const { return __ldcs(rec + c * n + r); }
+    __device__ __forceinline__ double aat(int c, int64_t r) const { return __ldg(arec + r * kAoS + c); }
+    // column c of object r from the layout kA selects (true: refinement records)
+    template <bool kA>
+    __device__ __forceinline__ double col(int c, int64_t r) const { return kA ? aat(c, r) : at(c, r); }
 };
 
 // ---------------------------------------------------------------------------------------
@@ -364,23 +377,24 @@ __device__ __forceinline__ void kepler_solve(double M, double e, int cls, const 
 // plane: (x, y) -> (-y, x)) + dOmega z x r.
 // kClass: 0 = object known to be class 0 (lean path), -1 = any class
 // kJ2: 0 = two-body only, 1 = J2 secular only, -1 = per O.j2 (runtime, warp-uniform)
-template <bool kVel, int kClass = -1, int kJ2 = -1>
+// kA: read the refinement records (Orbits::arec, random access) instead of the columns
+template <bool kVel, int kClass = -1, int kJ2 = -1, bool kA = false>
 __device__ __forceinline__ void state(const Orbits& O, int64_t r, double t, double p[3], double v[3])
 {
-    const double e = O.at(kE, r);
-    const double M = mean_anomaly(O.at(kM0, r), O.at(kNm, r), t);
+    const double e = O.col<kA>(kE, r);
+    const double M = mean_anomaly(O.col<kA>(kM0, r), O.col<kA>(kNm, r), t);
     double E, sE, cE;
     if (kClass == 0) contour_core<4>(M, e, O, r, E, sE, cE);
-    else kepler_solve(M, e, O.cls[r], O, r, E, sE, cE);
+    else kepler_solve(M, e, kA ? (int)O.aat(kAoSCls, r) : (int)O.cls[r], O, r, E, sE, cE);
     double x = cE - e, y = sE;              // coefficients of aP and bQ
     double vx = -sE, vy = cE;               // velocity coefficients (times n/(1 - e cos E))
     const bool j2 = kJ2 == 1 || (kJ2 == -1 && O.j2);
     double sO = 0.0, cO = 1.0, dOm = 0.0, dw = 0.0, ba = 1.0, ab = 1.0;
     if (j2) {
-        dOm = O.at(kDOm, r);
-        dw = O.at(kDw, r);
-        ba = O.at(kBA, r);
-        ab = O.at(kAB, r);
+        dOm = O.col<kA>(kDOm, r);
+        dw = O.col<kA>(kDw, r);
+        ba = O.col<kA>(kBA, r);
+        ab = O.col<kA>(kAB, r);
         double sw, cw;
         sincos_fast(dw * t, sw, cw);
         sincos_fast(dOm * t, sO, cO);
@@ -393,12 +407,12 @@ __device__ __forceinline__ void state(const Orbits& O, int64_t r, double t, doub
             vy = vyr;
         }
     }
-    const double ap[3] = {O.at(kAPx, r), O.at(kAPy, r), O.at(kAPz, r)};
-    const double bq[3] = {O.at(kBQx, r), O.at(kBQy, r), O.at(kBQz, r)};
+    const double ap[3] = {O.col<kA>(kAPx, r), O.col<kA>(kAPy, r), O.col<kA>(kAPz, r)};
+    const double bq[3] = {O.col<kA>(kBQx, r), O.col<kA>(kBQy, r), O.col<kA>(kBQz, r)};
 #pragma unroll
     for (int c = 0; c < 3; ++c) p[c] = fma(x, ap[c], y * bq[c]);
     if (kVel) {
-        const double k = O.at(kNm, r) / fma(-e, cE, 1.0);
+        const double k = O.col<kA>(kNm, r) / fma(-e, cE, 1.0);
         if (j2) {
             // domega h x r: the in-plane vector (X, Y) in unit (P, Q) axes turns to (-Y, X);
             // in (aP, bQ) coefficients: (-(b/a) y, (a/b) x)

@@ -80,8 +80,8 @@ struct RefineParams {
 cudaError_t launch_classify(const Elements& el, int64_t n, uint32_t* key, uint32_t* idx,
                             unsigned long long* n0, int min_cls, cudaStream_t st, LaunchCount& lc);
 cudaError_t launch_build_records(const Elements& el, const uint32_t* perm, int64_t n,
-                                 double* rec, uint8_t* cls, int j2, int min_cls, cudaStream_t st,
-                                 LaunchCount& lc);
+                                 double* rec, double* arec, uint8_t* cls, int j2, int min_cls,
+                                 cudaStream_t st, LaunchCount& lc);
 cudaError_t launch_propagate_out(const cdk::Orbits& O, const uint32_t* perm, const double* t,
                                  int64_t nt, double* xyz, double* vxyz, cudaStream_t st,
                                  LaunchCount& lc);

@@ -79,7 +79,8 @@ __global__ void k_classify(Elements el, int64_t n, uint32_t* key, uint32_t* idx,
 }
 
 __global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, int64_t n,
-                                double* __restrict__ rec, uint8_t* __restrict__ cls, int j2, int min_cls)
+                                double* __restrict__ rec, double* __restrict__ arec,
+                                uint8_t* __restrict__ cls, int j2, int min_cls)
 {
     const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (r >= n) return;
@@ -99,7 +100,11 @@ __global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, 
     sincos(0.5 * nu0, &sh, &ch);
     const double E0 = 2.0 * atan2(sqrt(1.0 - e) * sh, sqrt(1.0 + e) * ch);
     const double M0 = E0 - e * sin(E0);
-    auto put = [&](int c, double v) { rec[c * n + r] = v; };
+    // column-major (the per-step build) and object-major (the refinement's gathers)
+    auto put = [&](int c, double v) {
+        rec[c * n + r] = v;
+        arec[r * kAoS + c] = v;
+    };
     put(kM0, M0);
     const double n0 = sqrt(kMu / (a * a * a));
     if (j2) {
@@ -124,6 +129,7 @@ __global__ void k_build_records(Elements el, const uint32_t* __restrict__ perm, 
     put(kQper, a * (1.0 - e));
     const int cl = max(ecc_class(e), min_cls);
     cls[r] = (uint8_t)cl;
+    arec[r * kAoS + kAoSCls] = (double)cl;
 }
 
 __global__ void k_propagate_out(Orbits O, const uint32_t* __restrict__ perm,
@@ -152,9 +158,10 @@ cudaError_t launch_classify(const Elements& el, int64_t n, uint32_t* key, uint32
 }
 
 cudaError_t launch_build_records(const Elements& el, const uint32_t* perm, int64_t n, double* rec,
-                                 uint8_t* cls, int j2, int min_cls, cudaStream_t st, LaunchCount& lc)
+                                 double* arec, uint8_t* cls, int j2, int min_cls, cudaStream_t st,
+                                 LaunchCount& lc)
 {
-    k_build_records<<<blocks_for(n, 128), 128, 0, st>>>(el, perm, n, rec, cls, j2, min_cls);
+    k_build_records<<<blocks_for(n, 128), 128, 0, st>>>(el, perm, n, rec, arec, cls, j2, min_cls);
     lc.bump();
     return cudaGetLastError();
 }
@@ -894,7 +901,12 @@ __global__ void __launch_bounds__(256) k_prefilter(Orbits O, RefineParams P, con
         grid_refine_item(O, P, q[idx], 0u, w, wcap, n_work, out, ocap, ctrl);
 }
 
-__global__ void __launch_bounds__(128) k_brent(Orbits O, RefineParams P, const Work* __restrict__ w,
+// 5 blocks per SM (<= 102 registers; the evaluations are non-inlined calls): refine per step
+// 99 -> 82 us at 8M objects, 1.76 -> 1.45 us at 1M, hybrid 102 -> 97 us (1 / 3 / 4 / 6 / 8 blocks measured)
+#ifndef CD_BRENT_MINB
+#define CD_BRENT_MINB 5
+#endif
+__global__ void __launch_bounds__(128, CD_BRENT_MINB) k_brent(Orbits O, RefineParams P, const Work* __restrict__ w,
                                                const unsigned long long* n_work, size_t wcap,
                                                Conj* __restrict__ out, size_t ocap, Ctrl* ctrl)
 {

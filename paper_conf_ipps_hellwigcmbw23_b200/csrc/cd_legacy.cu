@@ -166,8 +166,8 @@ __global__ void __launch_bounds__(128) k_legacy_search(Orbits O, LegacyParams P,
                 continue;
             }
             double ri[3], vi[3], rj[3], vj[3];
-            state<true>(O, it.i, tk, ri, vi);
-            state<true>(O, it.j, tk, rj, vj);
+            state<true, -1, -1, true>(O, it.i, tk, ri, vi);
+            state<true, -1, -1, true>(O, it.j, tk, rj, vj);
             const double dv[3] = {vi[0] - vj[0], vi[1] - vj[1], vi[2] - vj[2]};
             if (dv[0] * dv[0] + dv[1] * dv[1] + dv[2] * dv[2] < 1e-18) continue;   // degenerate
             double x, fx;
