@@ -323,8 +323,9 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
 // a5-a6: neighbour scan, one thread per (object, step).
 //  (1) own cell: walk the object's own list successors -- every same-cell pair is seen exactly
 //      once, by the later-inserted object (no probe needed);
-//  (2) other cells: half-shell mode (L < 2 g_c, the paper's cell g_c) probes the 13
-//      positive half-shell neighbours -- each unordered pair of cells of a 3x3x3 block once;
+//  (2) other cells: half-shell mode (L < 2 g_c, the paper's cell g_c) probes those of
+//      the 13 positive half-shell neighbours -- each unordered pair of cells of a 3x3x3 block once
+//      -- that lie within reach of the object (halfshell_reach);
 //      ball mode (L >= 2 g_c) probes those of the 0-7 other cells overlapping |x - p| < g_c
 //      that lie in the positive (lexicographic) half-space of the own cell -- a pair in two
 //      cells is seen only from the smaller cell.  Each probe first tests the occupancy bitmap
@@ -337,6 +338,28 @@ __constant__ int8_t kHalfShell[14][3] = {
     {1, -1, -1}, {1, -1, 0}, {1, -1, 1}, {1, 0, -1}, {1, 0, 0}, {1, 0, 1}, {1, 1, -1}, {1, 1, 0}, {1, 1, 1},
     {0, 1, -1}, {0, 1, 0}, {0, 1, 1},
     {0, 0, 1}};
+
+// Half-shell offsets o = 1..13 whose cell can hold a point within the reach of p: the squared
+// distance from p to the cell, per axis 0 (same layer), fr^2 (offset -1) or (1 - fr)^2 (+1) in
+// cell units, below rl^2 (rl = reach / L).  Conservative like ball mode: reach = g_c (1 + 1e-9) +
+// 1e-9 km exceeds the rounding of fr by orders of magnitude.  (Offsets in kHalfShell's order.)
+__device__ __forceinline__ uint32_t halfshell_reach(const double fr[3], double rl)
+{
+#ifdef CD_NO_HS_PRUNE
+    return 0x3FFEu;
+#endif
+    const double r2 = rl * rl;
+    const double x1 = (1.0 - fr[0]) * (1.0 - fr[0]);
+    const double ys[3] = {fr[1] * fr[1], 0.0, (1.0 - fr[1]) * (1.0 - fr[1])};
+    const double zs[3] = {fr[2] * fr[2], 0.0, (1.0 - fr[2]) * (1.0 - fr[2])};
+    uint32_t m = 0;
+#pragma unroll
+    for (int o = 1; o <= 9; ++o) m |= (x1 + ys[(o - 1) / 3] + zs[(o - 1) % 3] < r2 ? 1u : 0u) << o;
+#pragma unroll
+    for (int o = 10; o <= 12; ++o) m |= (ys[2] + zs[o - 10] < r2 ? 1u : 0u) << o;
+    m |= (zs[2] < r2 ? 1u : 0u) << 13;
+    return m;
+}
 
 // Warp-level candidate staging (role-C warps of k_step, GridGeom::stage): each warp appends its
 // candidates to its own slice of a shared buffer with a shared-memory atomic and flushes them to
@@ -439,13 +462,14 @@ __device__ __forceinline__ void do_scan(const GridGeom& g, const GridTab& tab,
     // (2) other cells
     const uint32_t hx0 = (uint32_t)c[0] * kHX, hy0 = (uint32_t)c[1] * kHY, hz0 = (uint32_t)c[2] * kHZ;
     if (g.halfshell) {
+        const uint32_t reach = g.raw ? 0x3FFEu : halfshell_reach(fr, g.reach * g.inv_cell);   // (raw counts: the paper's 27 cells)
         uint32_t hit = 0;
 #pragma unroll
         for (int o = 1; o < 14; ++o) {
             const uint32_t hb = bit_mix((hx0 + (uint32_t)kHalfShell[o][0] * kHX) ^
                                         (hy0 + (uint32_t)kHalfShell[o][1] * kHY) ^
                                         (hz0 + (uint32_t)kHalfShell[o][2] * kHZ)) & bmask;
-            hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << o;
+            if ((reach >> o) & 1u) hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << o;
         }
         while (hit) {
             const int o = __ffs(hit) - 1;
@@ -542,9 +566,11 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
         // 3x3x3 block differ pairwise in (c mod 4) on some axis, so with superblock buckets they
         // never share a bucket: a colliding cell in the own bucket is never a neighbour (its
         // entries fail the distance test), and no pair is seen from two buckets.
+        const uint32_t reach = g.raw ? 0x3FFEu : halfshell_reach(fr, g.reach * g.inv_cell);   // (raw counts: the paper's 27 cells)
         uint32_t hit = 0;
 #pragma unroll
         for (int o = 1; o < 14; ++o) {
+            if (!((reach >> o) & 1u)) continue;
             const uint32_t h = __ldg(heads + chain_bucket(c[0] + kHalfShell[o][0], c[1] + kHalfShell[o][1],
                                                           c[2] + kHalfShell[o][2], hmask));
             hit |= (head_index(h, epoch) != kNil ? 1u : 0u) << o;
@@ -717,13 +743,18 @@ __device__ __forceinline__ void do_scan_csr(const GridGeom& g, const GridTab& ta
     const uint32_t hx0 = (uint32_t)c[0] * kHX, hy0 = (uint32_t)c[1] * kHY, hz0 = (uint32_t)c[2] * kHZ;
     uint32_t st, cnt;
     if (g.halfshell) {
+        // the lanes of a crowded cell are adjacent and walk the same neighbour ranges in lockstep:
+        // the warp's union of the reach masks keeps them converged (per-lane masks diverged
+        // them -- 8M hybrid scan 10.1 -> 15.0 ms per coarse step)
+        const uint32_t reach = g.raw ? 0x3FFEu
+                                     : __reduce_or_sync(__activemask(), halfshell_reach(fr, g.reach * g.inv_cell));
         uint32_t hit = 0;
 #pragma unroll
         for (int o = 1; o < 14; ++o) {
             const uint32_t hb = bit_mix((hx0 + (uint32_t)kHalfShell[o][0] * kHX) ^
                                         (hy0 + (uint32_t)kHalfShell[o][1] * kHY) ^
                                         (hz0 + (uint32_t)kHalfShell[o][2] * kHZ)) & bmask;
-            hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << o;
+            if ((reach >> o) & 1u) hit |= ((__ldg(bits + (hb >> 5)) >> (hb & 31)) & 1u) << o;
         }
         while (hit) {
             const int o = __ffs(hit) - 1;
