@@ -250,7 +250,11 @@ cudaError_t launch_conj_to_global(const Conj* in, size_t n, const uint32_t* perm
 // Grid structures (cd_options.grid_table): kOpen = the paper's open-addressing map with per-cell
 // lists, kChained = chained spatial hash, kCsr = open-addressing map of per-cell counts plus a
 // counting sort of the entries by cell (sort + segment: each cell's objects contiguous).
-enum GridKind : int { kOpen = 0, kChained = 1, kCsr = 2 };
+enum GridKind : int { kOpen = 0, kChained = 1, kCsr = 2, kChainedBall = 3 };
+// kChainedBall: the chained grid compiled for ball-mode scans only (the grid variant's hot
+// instance: the half-shell branch's code had cost its ball-mode scan 3 % -- 59.7 vs 61.6 us per
+// 1M-object step -- through register allocation)
+__host__ __device__ constexpr bool is_chained(int k) { return k == kChained || k == kChainedBall; }
 
 // CSR grid insert: claim the cell's slot (128-bit CAS from a stale slot to {key, tag | 1}) or
 // count the object into it (64-bit atomicAdd on the head word; count in the low 32 bits).
@@ -294,7 +298,7 @@ __device__ __forceinline__ void do_build(const Orbits& O, const GridGeom& g, con
         const uint32_t hb = bit_hash(c[0], c[1], c[2]) & tab.bmask;
         atomicOr(tab.bits + (size_t)s * tab.bwords + (hb >> 5), 1u << (hb & 31));
         next = grid_count(tab.slots + (size_t)s * (mask + 1), mask, pack_key(c[0], c[1], c[2]), tag, &ctag);
-    } else if (kGrid == kChained && cell_of(g, p, c)) {
+    } else if (is_chained(kGrid) && cell_of(g, p, c)) {
         ctag = cell_tag(c[0], c[1], c[2]);
         // chained spatial hash: push onto the list of bucket hash(cell) -- one atomic exchange;
         // heads hold index + 1 (0 = empty bucket)
@@ -544,6 +548,7 @@ __device__ __forceinline__ void walk_bucket_tag(const GridGeom& g, const Entry* 
     }
 }
 
+template <bool kBallOnly>
 __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab& tab,
                                                 const Entry* __restrict__ ents, int64_t n, int64_t k0,
                                                 int s, int64_t r, uint32_t epoch, Cand* __restrict__ q,
@@ -560,7 +565,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
     if (!cell_of(g, p, c, fr)) return;
     // own bucket: successors only, every pair once (by the later-inserted object)
     walk(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
-    if (g.halfshell) {
+    if (!kBallOnly && g.halfshell) {
         // L < 2 g_c: the 13 half-shell neighbour cells (each unordered pair of cells of a 3x3x3
         // block once, as in do_scan), only the probed cell's entries (tag).  The 27 cells of a
         // 3x3x3 block differ pairwise in (c mod 4) on some axis, so with superblock buckets they
@@ -804,7 +809,7 @@ __device__ __forceinline__ void do_scan_csr(const GridGeom& g, const GridTab& ta
 #define CD_OPEN_MINB 6
 #endif
 template <int kGrid, int kJ2>
-__global__ void __launch_bounds__(256, kGrid == kChained ? CD_STEP_MINB : CD_OPEN_MINB) k_step(StepArgs a)
+__global__ void __launch_bounds__(256, is_chained(kGrid) ? CD_STEP_MINB : CD_OPEN_MINB) k_step(StepArgs a)
 {
     const uint32_t bx = blockIdx.x;
     const uint32_t nbA = (uint32_t)a.nbA, nbB = (uint32_t)a.nbB, nbC = (uint32_t)a.nbC;
@@ -837,7 +842,7 @@ __global__ void __launch_bounds__(256, kGrid == kChained ? CD_STEP_MINB : CD_OPE
         const int64_t nth = a.nCblocks * 256;
         const int64_t nw4 = (int64_t)a.zero_depth * a.zero_bits_words / 4;
         uint4* zb = reinterpret_cast<uint4*>(a.zero_bits);
-        if (kGrid != kChained)   // chained heads are epoch-tagged: nothing to clear
+        if (!is_chained(kGrid))   // chained heads are epoch-tagged: nothing to clear
             for (int64_t i = tid; i < nw4; i += nth) zb[i] = make_uint4(0u, 0u, 0u, 0u);
         if (a.scan_B == 0) return;
         const int s = (int)(b3 / nbC);
@@ -852,8 +857,8 @@ __global__ void __launch_bounds__(256, kGrid == kChained ? CD_STEP_MINB : CD_OPE
             __syncwarp();
         }
         if (r < a.O.n) {
-            if (kGrid == kChained)
-                do_scan_chained(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
+            if (is_chained(kGrid))
+                do_scan_chained<kGrid == kChainedBall>(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
                                 a.qcap, a.ctrl);
             else if (kGrid == kCsr)
                 do_scan_csr(a.g, a.scan_tab, a.scan_start, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r,
@@ -900,7 +905,8 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
         return launch_ex(k_step<kOpen, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
     }
     if (a.chained)
-        return launch_ex(k_step<kChained, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, a.pdl != 0, a);
+        return launch_ex(a.g.halfshell ? k_step<kChained, 0> : k_step<kChainedBall, 0>, dim3((unsigned)blocks),
+                         dim3(256), smem, st, win, a.pdl != 0, a);
     if (a.csr)
         return launch_ex(k_step<kCsr, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
     return launch_ex(k_step<kOpen, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
