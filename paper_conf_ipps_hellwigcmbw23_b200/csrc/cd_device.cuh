@@ -250,8 +250,7 @@ __host__ __device__ constexpr int series_terms(int N)
 }
 
 template <int N>
-__device__ __forceinline__ void contour_core(double M, double e, const Orbits& O, int64_t r,
-                                             double& E, double& sE, double& cE)
+__device__ __forceinline__ void contour_core(double M, double e, double& E, double& sE, double& cE)
 {
     const double rho = 0.5 * e;
     const bool lower = M < kPi;
@@ -347,16 +346,15 @@ __device__ __forceinline__ void contour_core(double M, double e, const Orbits& O
 }
 
 // Eccentricity-class dispatch (objects are sorted by class, so warps are uniform).
-__device__ __forceinline__ void kepler_solve(double M, double e, int cls, const Orbits& O,
-                                             int64_t r, double& E, double& sE, double& cE)
+__device__ __forceinline__ void kepler_solve(double M, double e, int cls, double& E, double& sE, double& cE)
 {
     switch (cls) {
-    case 0: contour_core<4>(M, e, O, r, E, sE, cE); break;
-    case 1: contour_core<6>(M, e, O, r, E, sE, cE); break;
-    case 2: contour_core<8>(M, e, O, r, E, sE, cE); break;
-    case 3: contour_core<12>(M, e, O, r, E, sE, cE); break;
+    case 0: contour_core<4>(M, e, E, sE, cE); break;
+    case 1: contour_core<6>(M, e, E, sE, cE); break;
+    case 2: contour_core<8>(M, e, E, sE, cE); break;
+    case 3: contour_core<12>(M, e, E, sE, cE); break;
     default:
-        contour_core<16>(M, e, O, r, E, sE, cE);
+        contour_core<16>(M, e, E, sE, cE);
         if (e > 0.8) {   // Newton polish of the contour estimate (R15)
             for (int it = 0; it < 8; ++it) {
                 const double dE = (E - e * sE - M) * rcp_fast(1.0 - e * cE);
@@ -366,6 +364,15 @@ __device__ __forceinline__ void kepler_solve(double M, double e, int cls, const 
             }
         }
     }
+}
+
+// One out-of-line copy of the class dispatch for the refinement (state<..., kA = true>): Brent and
+// the polish evaluate two states per call site, and inlining the five Contour instances at each
+// had made k_brent instruction-cache bound (ncu at 8M objects: 9.9 no-instruction stalls per
+// issue).
+static __device__ __noinline__ void kepler_solve_ool(double M, double e, int cls, double& E, double& sE, double& cE)
+{
+    kepler_solve(M, e, cls, E, sE, cE);
 }
 
 // Position (and velocity) of object r at time t.
@@ -384,8 +391,9 @@ __device__ __forceinline__ void state(const Orbits& O, int64_t r, double t, doub
     const double e = O.col<kA>(kE, r);
     const double M = mean_anomaly(O.col<kA>(kM0, r), O.col<kA>(kNm, r), t);
     double E, sE, cE;
-    if (kClass == 0) contour_core<4>(M, e, O, r, E, sE, cE);
-    else kepler_solve(M, e, kA ? (int)O.aat(kAoSCls, r) : (int)O.cls[r], O, r, E, sE, cE);
+    if (kClass == 0) contour_core<4>(M, e, E, sE, cE);
+    else if (kA) kepler_solve_ool(M, e, (int)O.aat(kAoSCls, r), E, sE, cE);
+    else kepler_solve(M, e, (int)O.cls[r], E, sE, cE);
     double x = cE - e, y = sE;              // coefficients of aP and bQ
     double vx = -sE, vy = cE;               // velocity coefficients (times n/(1 - e cos E))
     const bool j2 = kJ2 == 1 || (kJ2 == -1 && O.j2);

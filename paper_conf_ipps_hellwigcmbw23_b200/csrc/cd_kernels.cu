@@ -938,10 +938,11 @@ __global__ void __launch_bounds__(256) k_prefilter(Orbits O, RefineParams P, con
         grid_refine_item(O, P, q[idx], 0u, w, wcap, n_work, out, ocap, ctrl);
 }
 
-// 5 blocks per SM (<= 102 registers; the evaluations are non-inlined calls): refine per step
-// 99 -> 82 us at 8M objects, 1.76 -> 1.45 us at 1M, hybrid 102 -> 97 us (1 / 3 / 4 / 6 / 8 blocks measured)
+// 4 blocks per SM (<= 128 registers; the evaluations and the Kepler solve are out-of-line calls):
+// refine per step 99 -> 61 us at 8M objects, 1.76 -> 1.29 us at 1M, hybrid 102 -> 91 us (1 / 3 / 4 /
+// 5 / 6 / 8 blocks measured, profiles/round2_brent_minb.txt)
 #ifndef CD_BRENT_MINB
-#define CD_BRENT_MINB 5
+#define CD_BRENT_MINB 4
 #endif
 __global__ void __launch_bounds__(128, CD_BRENT_MINB) k_brent(Orbits O, RefineParams P, const Work* __restrict__ w,
                                                const unsigned long long* n_work, size_t wcap,
