@@ -593,11 +593,13 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
         uint32_t hit = 0;
 #pragma unroll
         for (int o = 1; o < 14; ++o) {
-            if (!((reach >> o) & 1u)) continue;
+            // (every head loaded, the unreachable ones discarded: branch-free, so the 13 loads are
+            // in flight together)
             const uint32_t h = __ldg(heads + chain_bucket(c[0] + kHalfShell[o][0], c[1] + kHalfShell[o][1],
                                                           c[2] + kHalfShell[o][2], hmask));
             hit |= (head_index(h, epoch) != kNil ? 1u : 0u) << o;
         }
+        hit &= reach;
         while (hit) {
             const int o = __ffs(hit) - 1;
             hit &= hit - 1;
