@@ -102,7 +102,10 @@ def test_candidates_ragged_sizes(n, steps, d):
                                 dict(cell_factor=3.7), dict(batch_object_steps=1),
                                 dict(round_steps=7), dict(batch_object_steps=10 ** 7),
                                 dict(grid_table=3), dict(grid_table=3, cell_factor=1.0),
-                                dict(grid_table=3, batch_object_steps=1), dict(grid_table=3, round_steps=5)])
+                                dict(grid_table=3, batch_object_steps=1), dict(grid_table=3, round_steps=5),
+                                dict(grid_table=2, cell_factor=1.5, grid_origin=(-3e3, 7.5, 1e4)),
+                                dict(grid_table=2, cell_factor=1.9, grid_origin=(11.0, -2.5, 0.75)),
+                                dict(grid_table=1, cell_factor=1.9)])
 def test_candidates_invariance(kw):
     pop = _mix(8000, 5)
     d = 20.0
@@ -110,6 +113,27 @@ def test_candidates_invariance(kw):
     Ko = oracle.candidates_grid(pop, 0.0, 59.0, 1.0, gc)
     Kg = cds.candidates(pop, 0.0, 59.0, 1.0, d, **kw)
     parity.compare_candidates(pop, Kg, Ko, 0.0, 1.0, gc)
+
+
+@pytest.mark.parametrize("table", [1, 2, 3])
+def test_halfshell_reach_swarm(table):
+    """Half-shell scans skip the neighbour cells out of reach of the object (halfshell_reach):
+    a compact swarm puts thousands of pairs across cell faces, edges and corners at distances
+    around g_c; every cell edge in half-shell mode (g_c <= L < 2 g_c) must give the brute-force
+    candidate set."""
+    rng = np.random.default_rng(21)
+    n = 2500
+    pop = {"a": 7000.0 + rng.uniform(-40, 40, n), "e": rng.uniform(0, 2e-3, n),
+           "inc": 0.9 + rng.normal(0, 4e-3, n), "raan": 1.0 + rng.normal(0, 4e-3, n),
+           "argp": rng.uniform(0, 0.2, n), "nu0": rng.uniform(0, 0.2, n)}
+    d, dt = 20.0, 1.0
+    gc = oracle.cell_size(d, dt)
+    Ko = oracle.candidates_brute(pop, 0.0, 4.0, dt, gc)
+    assert len(Ko) > 50000
+    for cf, org in ((1.0, (0.0, 0.0, 0.0)), (1.0, (13.1, -7.7, 2.9)), (1.3, (5.0, 5.0, 5.0)),
+                    (1.999, (-1.0, 2.0, -3.0))):
+        Kg = cds.candidates(pop, 0.0, 4.0, dt, d, cell_factor=cf, grid_origin=org, grid_table=table)
+        parity.compare_candidates(pop, Kg, Ko, 0.0, dt, gc)
 
 
 def test_worst_case_colocated_and_overflow_retry():
