@@ -21,7 +21,38 @@ struct __align__(128) HOrbit {   // one 128-byte line per object (compact gather
 };
 static_assert(sizeof(HOrbit) == 128, "HOrbit must be one 128-byte line");
 
-__device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o)
+// The hybrid filter's stage 1 (apogee/perigee, coplanarity, orbit path) reads only a, e and the
+// perifocal unit vectors: one 64-byte line per object (64 MB at 1M objects, L2-resident), loaded
+// whole into registers; q, Q, p and h are derived there with horbit's own expressions (so the
+// values are bit-identical to HOrbit's).
+struct __align__(64) HHot {
+    double a, e, P[3], Qv[3];
+};
+static_assert(sizeof(HHot) == 64, "HHot must be one 64-byte line");
+
+// the HOrbit fields stage 1 uses, in registers
+struct HGeo {
+    double e, q, Q, p;
+    double P[3], Qv[3], h[3];
+};
+__device__ __forceinline__ HGeo geo_of(const HHot& o)
+{
+    HGeo g;
+    g.e = o.e;
+    g.q = o.a * (1.0 - o.e);
+    g.Q = o.a * (1.0 + o.e);
+    g.p = o.a * (1.0 - o.e) * (1.0 + o.e);
+    for (int c = 0; c < 3; ++c) {
+        g.P[c] = o.P[c];
+        g.Qv[c] = o.Qv[c];
+    }
+    g.h[0] = g.P[1] * g.Qv[2] - g.P[2] * g.Qv[1];
+    g.h[1] = g.P[2] * g.Qv[0] - g.P[0] * g.Qv[2];
+    g.h[2] = g.P[0] * g.Qv[1] - g.P[1] * g.Qv[0];
+    return g;
+}
+
+__device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o, HHot& hot)
 {
     const double ap[3] = {O.at(kAPx, r), O.at(kAPy, r), O.at(kAPz, r)};
     const double bq[3] = {O.at(kBQx, r), O.at(kBQy, r), O.at(kBQz, r)};
@@ -41,6 +72,12 @@ __device__ __forceinline__ void horbit(const Orbits& O, int64_t r, HOrbit& o)
     o.nm = O.at(kNm, r);
     o.M0 = O.at(kM0, r);
     o.inm = 1.0 / o.nm;
+    hot.a = a;
+    hot.e = o.e;
+    for (int c = 0; c < 3; ++c) {
+        hot.P[c] = o.P[c];
+        hot.Qv[c] = o.Qv[c];
+    }
 }
 
 // Divisions are reciprocal estimates refined to full precision (rcp_fast: two Newton steps) times
@@ -66,7 +103,8 @@ __device__ __forceinline__ double mean_of_true_cs(double c, double s, double e)
 // radius range over the true anomalies (f - a, f + a) of node `sg` (+1: f, -1: f + pi), a < pi/2:
 // the ends r = p / (1 + e cos(f -+ a)), widened to the perigee radius if the interval contains
 // f = 0 (cos f >= cos a) and to the apogee radius if it contains f = pi (-cos f >= cos a)
-__device__ __forceinline__ void radius_range(const HOrbit& o, const NodeGeom& g, double sg,
+template <typename R>
+__device__ __forceinline__ void radius_range(const R& o, const NodeGeom& g, double sg,
                                              double& rmin, double& rmax)
 {
     const double cf = sg * g.cf, sf = sg * g.sf;
@@ -95,7 +133,8 @@ __device__ __forceinline__ void node_window(const HOrbit& o, const NodeGeom& g, 
 // of each orbit.
 //   AP:        exclude iff max(q_A, q_B) - min(Q_A, Q_B) > d
 //   coplanar:  s_X = d / (q_X sin D) >= 1 for A or B, or q_A cos(asin s_A) + q_B cos(asin s_B) <= d
-__device__ __forceinline__ int pair_geometry(const HOrbit& A, const HOrbit& B, double d,
+template <typename R>
+__device__ __forceinline__ int pair_geometry(const R& A, const R& B, double d,
                                              bool& coplanar, NodeGeom& gA, NodeGeom& gB)
 {
     if (fmax(A.q, B.q) - fmin(A.Q, B.Q) > d) return 1;
@@ -129,7 +168,8 @@ __device__ __forceinline__ int pair_geometry(const HOrbit& A, const HOrbit& B, d
 
 // orbit-path filter at node sg (+1 / -1): true iff the radial ranges of A and B over their node
 // windows are more than d apart (|r_A - r_B| >= ||r_A| - |r_B||)
-__device__ __forceinline__ bool node_closed(const HOrbit& A, const HOrbit& B, double d,
+template <typename R>
+__device__ __forceinline__ bool node_closed(const R& A, const R& B, double d,
                                             const NodeGeom& gA, const NodeGeom& gB, double sg)
 {
     double rAl, rAh, rBl, rBh;

@@ -33,8 +33,10 @@ __global__ void k_build_hrec(Orbits O, HOrbit* __restrict__ hr)
     const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (r >= O.n) return;
     HOrbit o;
-    horbit(O, r, o);
+    HHot h;
+    horbit(O, r, o, h);
     hr[r] = o;
+    reinterpret_cast<HHot*>(hr + O.n)[r] = h;   // the stage-1 lines follow the full records
 }
 
 #ifndef CD_FILTER_MINB
@@ -111,6 +113,7 @@ __global__ void __launch_bounds__(256, CD_FILTER_MINB) k_hybrid_filter(Orbits O,
 {
     __shared__ uint64_t s_fq[8][kFQ];   // per warp: (candidate index << 2) | open-node mask
     const HOrbit* __restrict__ hr = static_cast<const HOrbit*>(P.hrec);
+    const HHot* __restrict__ hot = reinterpret_cast<const HHot*>(hr + O.n);
     unsigned long long nc = ctrl->n_cand;
     if (nc > qcap) nc = qcap;
     const unsigned lane = threadIdx.x & 31u, wid = threadIdx.x >> 5;
@@ -123,13 +126,12 @@ __global__ void __launch_bounds__(256, CD_FILTER_MINB) k_hybrid_filter(Orbits O,
         if (idx < nc) {
             const Cand cd = q[idx];
             const double d = P.d;
-            // apogee / perigee first, from 16 bytes of each record
-            if (fmax(hr[cd.i].q, hr[cd.j].q) - fmin(hr[cd.i].Q, hr[cd.j].Q) > d) {
+            const HHot ha = hot[cd.i], hb = hot[cd.j];   // one 64-byte line each
+            // apogee / perigee first
+            if (fmax(ha.a * (1.0 - ha.e), hb.a * (1.0 - hb.e)) - fmin(ha.a * (1.0 + ha.e), hb.a * (1.0 + hb.e)) > d) {
                 count1(&ctrl->n_ap);
             } else {
-                // records by reference: fields are loaded where used
-                const HOrbit& A = hr[cd.i];
-                const HOrbit& B = hr[cd.j];
+                const HGeo A = geo_of(ha), B = geo_of(hb);
                 bool coplanar;
                 NodeGeom gA, gB;
                 if (pair_geometry(A, B, d, coplanar, gA, gB)) {   // apogee / perigee
@@ -161,7 +163,7 @@ __global__ void __launch_bounds__(256, CD_FILTER_MINB) k_hybrid_filter(Orbits O,
     if (lane < qt - qh) filter_windows(hr, P, q, fq[(qh + lane) % kFQ], w, wcap, n_work, ctrl);
 }
 
-size_t hybrid_record_bytes() { return sizeof(HOrbit); }
+size_t hybrid_record_bytes() { return sizeof(HOrbit) + sizeof(HHot); }
 
 cudaError_t launch_build_hybrid_records(const Orbits& O, void* hrec, cudaStream_t st, LaunchCount& lc)
 {
