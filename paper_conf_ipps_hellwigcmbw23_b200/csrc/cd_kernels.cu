@@ -624,10 +624,10 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
     uint32_t hd[8];
 #pragma unroll
     for (int b = 1; b < 8; ++b)
-        hd[b] = ((valid >> b) & 1u)
-                    ? __ldg(heads + chain_bucket(c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0),
-                                                 c[2] + ((b & 4) ? d2 : 0), hmask))
-                    : 0u;
+        // every head loaded (branch-free, all in flight together), the invalid ones discarded:
+        // 59.4 -> 58.7 us per 1M-object step, 766 -> 759 us per 8M step
+        hd[b] = __ldg(heads + chain_bucket(c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0),
+                                           c[2] + ((b & 4) ? d2 : 0), hmask)) & (((valid >> b) & 1u) ? ~0u : 0u);
 #pragma unroll
     for (int b = 1; b < 8; ++b)
         if (hd[b])
