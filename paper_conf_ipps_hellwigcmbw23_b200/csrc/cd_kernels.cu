@@ -922,7 +922,8 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
     const size_t smem = a.g.stage ? sizeof(Cand) * kSCand : 0;   // candidate staging buffer
     if (a.O.j2) {   // J2 secular propagator: the rotation is compiled into its own instances
         if (a.chained)
-            return launch_ex(k_step<kChained, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, a.pdl != 0, a);
+            return launch_ex(a.g.halfshell ? k_step<kChained, 1> : k_step<kChainedBall, 1>, dim3((unsigned)blocks),
+                             dim3(256), smem, st, win, a.pdl != 0, a);
         if (a.csr)
             return launch_ex(k_step<kCsr, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
         return launch_ex(k_step<kOpen, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
