@@ -454,7 +454,8 @@ __device__ __forceinline__ void walk(const GridGeom& g, const Entry* __restrict_
 // queued) did not pay: 446 -> 451 us scan, 161 -> 165 us filter per step; 16 lanes per object,
 // one half-shell cell each (more loads in flight, 16x the per-lane set-up), 432 vs 282 us; and
 // fewer blocks per SM for a spill-free open-map instance (CD_OPEN_MINB 5 / 4 / 3: 48 / 61 / 61
-// registers), 301 / 356 / 354 vs 282 us -- occupancy outweighs the spills.
+// registers), 301 / 356 / 354 vs 282 us -- occupancy outweighs the spills (and more blocks win:
+// 8 per SM, 32 registers, for the half-shell instances, see CD_HALF_MINB / CD_OPEN_MINB).
 __device__ __forceinline__ void probe_cell(const GridGeom& g, const Slot* __restrict__ slots,
                                            uint64_t mask, uint32_t tag, int cx, int cy, int cz,
                                            const Entry* __restrict__ E, uint32_t r, const double p[3],
@@ -828,11 +829,23 @@ __device__ __forceinline__ void do_scan_csr(const GridGeom& g, const GridTab& ta
 #ifndef CD_STEP_MINB
 #define CD_STEP_MINB 6
 #endif
+// blocks per SM of the other instances (measured on the 1M hybrid's half-shell scan: 6 -> 8
+// blocks, i.e. 40 -> 32 registers with spills, 222 -> 213 us chained and 256 -> 229 us open
+// map; the crowded sort + segment grid at 8M prefers 6: 10.21 vs 10.31 ms)
 #ifndef CD_OPEN_MINB
-#define CD_OPEN_MINB 6
+#define CD_OPEN_MINB 8
+#endif
+#ifndef CD_CSR_MINB
+#define CD_CSR_MINB 6
 #endif
 template <int kGrid, int kJ2>
-__global__ void __launch_bounds__(256, is_chained(kGrid) ? CD_STEP_MINB : CD_OPEN_MINB) k_step(StepArgs a)
+#ifndef CD_HALF_MINB
+#define CD_HALF_MINB 8   // kChained: the half-shell (and J2 runtime) instance
+#endif
+__global__ void __launch_bounds__(256, kGrid == kChained     ? CD_HALF_MINB
+                                       : is_chained(kGrid) ? CD_STEP_MINB
+                                       : kGrid == kCsr     ? CD_CSR_MINB
+                                                           : CD_OPEN_MINB) k_step(StepArgs a)
 {
     const uint32_t bx = blockIdx.x;
     const uint32_t nbA = (uint32_t)a.nbA, nbB = (uint32_t)a.nbB, nbC = (uint32_t)a.nbC;
