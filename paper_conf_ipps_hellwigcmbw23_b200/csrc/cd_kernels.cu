@@ -963,7 +963,10 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
 //     discarded ("the minimum will be found when considering the neighboring
 //     interval"); otherwise it is reported iff its owner step is k and D < d.
 // ---------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) k_prefilter(Orbits O, RefineParams P, const Cand* __restrict__ q,
+#ifndef CD_PREFILTER_MINB
+#define CD_PREFILTER_MINB 3   // 1 / 3 / 4 blocks per SM: 8M refine 64.8 / 63.3 / 75.3 us per step, 1M 1.47 / 1.32 / 1.29
+#endif
+__global__ void __launch_bounds__(256, CD_PREFILTER_MINB) k_prefilter(Orbits O, RefineParams P, const Cand* __restrict__ q,
                                                    size_t qcap, Work* __restrict__ w, size_t wcap,
                                                    unsigned long long* n_work, Conj* __restrict__ out,
                                                    size_t ocap, Ctrl* ctrl)
