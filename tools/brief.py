@@ -8,4 +8,4 @@ for line in sys.stdin:
     except ValueError:
         print(line.rstrip())
         continue
-    print(f"table {d['table']} cell {d['cell']} resort {d['resort']}: scan {d['us_scan']:.1f} us, refine {d['us_refine']:.2f} us, cand {d['cand']}, conj {d['conj']}")
+    print(f"table {d['table']} cell {d['cell']} resort {d['resort']} rounds {d.get('rounds', 0)}: scan {d['us_scan']:.1f} us, refine {d['us_refine']:.2f} us, cand {d['cand']}, conj {d['conj']}")
