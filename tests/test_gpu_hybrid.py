@@ -56,6 +56,9 @@ def test_hybrid_shells_100k(table):
     pop, cfg, _ = popgen.make_config(3)
     res, st = _check(pop, 3600.0, 5400.0, 9.0, 2.0, grid_table=table)
     assert res["matched"] > 10 and st["hybrid_coplanar"] > 0
+    # the structure the call used: the default is the chained grid (half-shell scan of the
+    # reachable tagged buckets) at this density (< 3 candidates per object-step)
+    assert st["grid_table"] == {0: 2, 2: 2, 3: 3}[table]
 
 
 def test_hybrid_dense_and_coplanar():
