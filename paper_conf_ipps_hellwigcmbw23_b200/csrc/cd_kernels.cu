@@ -268,11 +268,13 @@ cudaError_t launch_conj_to_global(const Conj* in, size_t n, const uint32_t* perm
 // Grid structures (cd_options.grid_table): kOpen = the paper's open-addressing map with per-cell
 // lists, kChained = chained spatial hash, kCsr = open-addressing map of per-cell counts plus a
 // counting sort of the entries by cell (sort + segment: each cell's objects contiguous).
-enum GridKind : int { kOpen = 0, kChained = 1, kCsr = 2, kChainedBall = 3 };
+enum GridKind : int { kOpen = 0, kChained = 1, kCsr = 2, kChainedBall = 3, kChainedLean = 4 };
 // kChainedBall: the chained grid compiled for ball-mode scans only (the grid variant's hot
 // instance: the half-shell branch's code had cost its ball-mode scan 3 % -- 59.7 vs 61.6 us per
 // 1M-object step -- through register allocation)
-__host__ __device__ constexpr bool is_chained(int k) { return k == kChained || k == kChainedBall; }
+// kChainedLean: the half-shell chained scan without the shard band, slot map and raw counts
+// (test_pair<true>), chosen when none of them is active
+__host__ __device__ constexpr bool is_chained(int k) { return k == kChained || k == kChainedBall || k == kChainedLean; }
 
 // CSR grid insert: claim the cell's slot (128-bit CAS from a stale slot to {key, tag | 1}) or
 // count the object into it (64-bit atomicAdd on the head word; count in the low 32 bits).
@@ -398,20 +400,25 @@ extern __shared__ Cand s_cand[];
 __shared__ unsigned s_nw[8];
 __shared__ unsigned s_rw[8];   // per warp: pairs examined (emit_raw_counts)
 
+// kLean: no radial shard band, no slot -> id map, no raw counts (the hybrid's default call; a
+// separate instance so these features cost it no registers)
+template <bool kLean = false>
 __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_t j, const double p[3],
                                           const Entry& ej, uint32_t step, Cand* __restrict__ q,
                                           size_t qcap, Ctrl* ctrl)
 {
-    if (g.raw) atomicAdd(&s_rw[threadIdx.x >> 5], 1u);
+    if (!kLean && g.raw) atomicAdd(&s_rw[threadIdx.x >> 5], 1u);
     const double dx = p[0] - ej.x, dy = p[1] - ej.y, dz = p[2] - ej.z;
     if (fma(dx, dx, fma(dy, dy, dz * dz)) < g.gc2) {
         // radial shard: the pair belongs to the shard holding the smaller radius (identical
         // positions on every shard, so exactly one shard keeps it)
-        const double ra = fma(p[0], p[0], fma(p[1], p[1], p[2] * p[2]));
-        const double rb = fma(ej.x, ej.x, fma(ej.y, ej.y, ej.z * ej.z));
-        const double rm = fmin(ra, rb);
-        if (!(rm >= g.band_lo2 && rm < g.band_hi2)) return;
-        const uint32_t a = g.sig ? g.sig[r] : r, b = g.sig ? g.sig[j] : j;   // slots -> internal ids
+        if (!kLean) {
+            const double ra = fma(p[0], p[0], fma(p[1], p[1], p[2] * p[2]));
+            const double rb = fma(ej.x, ej.x, fma(ej.y, ej.y, ej.z * ej.z));
+            const double rm = fmin(ra, rb);
+            if (!(rm >= g.band_lo2 && rm < g.band_hi2)) return;
+        }
+        const uint32_t a = !kLean && g.sig ? g.sig[r] : r, b = !kLean && g.sig ? g.sig[j] : j;   // slots -> internal ids
         Cand cd;
         cd.i = a < b ? a : b;
         cd.j = a < b ? b : a;
@@ -428,6 +435,7 @@ __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_
     }
 }
 
+template <bool kLean = false>
 __device__ __forceinline__ void walk(const GridGeom& g, const Entry* __restrict__ E, uint32_t j,
                                      uint32_t r, const double p[3], bool only_greater, uint32_t step,
                                      Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
@@ -439,7 +447,7 @@ __device__ __forceinline__ void walk(const GridGeom& g, const Entry* __restrict_
             return;
         }
         const Entry ej = E[j];
-        if (!only_greater || j > r) test_pair(g, r, j, p, ej, step, q, qcap, ctrl);
+        if (!only_greater || j > r) test_pair<kLean>(g, r, j, p, ej, step, q, qcap, ctrl);
         j = ej.next;
     }
 }
@@ -549,6 +557,7 @@ __device__ __forceinline__ uint32_t head_index(uint32_t h, uint32_t epoch)
 // ball mode: bucket of the probed cell (tag ctag), which lies in the positive half-space of the
 // scanning object's cell -- only the probed cell's own entries count (a colliding neighbour
 // cell's entries are found by their own probe, so each pair is reported exactly once)
+template <bool kLean = false>
 __device__ __forceinline__ void walk_bucket_tag(const GridGeom& g, const Entry* __restrict__ E,
                                                 uint32_t h, uint32_t epoch, uint32_t ctag, uint32_t r,
                                                 const double p[3], uint32_t step,
@@ -562,12 +571,12 @@ __device__ __forceinline__ void walk_bucket_tag(const GridGeom& g, const Entry* 
             return;
         }
         const Entry ej = E[j];
-        if (ej.tag == ctag) test_pair(g, r, j, p, ej, step, q, qcap, ctrl);
+        if (ej.tag == ctag) test_pair<kLean>(g, r, j, p, ej, step, q, qcap, ctrl);
         j = ej.next;
     }
 }
 
-template <bool kBallOnly>
+template <bool kBallOnly, bool kLean = false>
 __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab& tab,
                                                 const Entry* __restrict__ ents, int64_t n, int64_t k0,
                                                 int s, int64_t r, uint32_t epoch, Cand* __restrict__ q,
@@ -586,8 +595,8 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
     double fr[3];
     if (!cell_of(g, p, c, fr)) return;
     // own bucket: successors only, every pair once (by the later-inserted object)
-    walk(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
-    if (!kBallOnly && g.halfshell) {
+    walk<kLean>(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
+    if (kLean || (!kBallOnly && g.halfshell)) {   // (the lean instance runs half-shell scans only)
         // L < 2 g_c: the 13 half-shell neighbour cells (each unordered pair of cells of a 3x3x3
         // block once, as in do_scan), only the probed cell's entries (tag).  The 27 cells of a
         // 3x3x3 block differ pairwise in (c mod 4) on some axis, so with superblock buckets they
@@ -608,7 +617,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
             const int o = __ffs(hit) - 1;
             hit &= hit - 1;
             const int cx = c[0] + kHalfShell[o][0], cy = c[1] + kHalfShell[o][1], cz = c[2] + kHalfShell[o][2];
-            walk_bucket_tag(g, E, __ldg(heads + chain_bucket(cx, cy, cz, hmask)), epoch, cell_tag(cx, cy, cz),
+            walk_bucket_tag<kLean>(g, E, __ldg(heads + chain_bucket(cx, cy, cz, hmask)), epoch, cell_tag(cx, cy, cz),
                             (uint32_t)r, p, step, q, qcap, ctrl);
         }
         return;
@@ -635,7 +644,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
 #pragma unroll
     for (int b = 1; b < 8; ++b)
         if (hd[b])
-            walk_bucket_tag(g, E, hd[b], epoch,
+            walk_bucket_tag<kLean>(g, E, hd[b], epoch,
                             cell_tag(c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0),
                                      c[2] + ((b & 4) ? d2 : 0)),
                             (uint32_t)r, p, step, q, qcap, ctrl);
@@ -842,7 +851,7 @@ template <int kGrid, int kJ2>
 #ifndef CD_HALF_MINB
 #define CD_HALF_MINB 8   // kChained: the half-shell (and J2 runtime) instance
 #endif
-__global__ void __launch_bounds__(256, kGrid == kChained     ? CD_HALF_MINB
+__global__ void __launch_bounds__(256, kGrid == kChained || kGrid == kChainedLean ? CD_HALF_MINB
                                        : is_chained(kGrid) ? CD_STEP_MINB
                                        : kGrid == kCsr     ? CD_CSR_MINB
                                                            : CD_OPEN_MINB) k_step(StepArgs a)
@@ -894,7 +903,7 @@ __global__ void __launch_bounds__(256, kGrid == kChained     ? CD_HALF_MINB
         }
         if (r < a.O.n) {
             if (is_chained(kGrid))
-                do_scan_chained<kGrid == kChainedBall>(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
+                do_scan_chained<kGrid == kChainedBall, kGrid == kChainedLean>(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
                                 a.qcap, a.ctrl);
             else if (kGrid == kCsr)
                 do_scan_csr(a.g, a.scan_tab, a.scan_start, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r,
@@ -933,6 +942,7 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
     if (blocks == 0) return cudaSuccess;
     lc.bump();
     const size_t smem = a.g.stage ? sizeof(Cand) * kSCand : 0;   // candidate staging buffer
+    const bool lean = !a.g.raw && !a.g.sig && a.g.band_lo2 == 0.0 && isinf(a.g.band_hi2);
     if (a.O.j2) {   // J2 secular propagator: the rotation is compiled into its own instances
         if (a.chained)
             return launch_ex(a.g.halfshell ? k_step<kChained, 1> : k_step<kChainedBall, 1>, dim3((unsigned)blocks),
@@ -942,7 +952,10 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
         return launch_ex(k_step<kOpen, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
     }
     if (a.chained)
-        return launch_ex(a.g.halfshell ? k_step<kChained, 0> : k_step<kChainedBall, 0>, dim3((unsigned)blocks),
+        return launch_ex(!a.g.halfshell ? k_step<kChainedBall, 0>
+                         : lean      ? k_step<kChainedLean, 0>
+                                     : k_step<kChained, 0>,
+                         dim3((unsigned)blocks),
                          dim3(256), smem, st, win, a.pdl != 0, a);
     if (a.csr)
         return launch_ex(k_step<kCsr, 0>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
