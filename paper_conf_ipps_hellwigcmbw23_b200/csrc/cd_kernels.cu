@@ -268,13 +268,13 @@ cudaError_t launch_conj_to_global(const Conj* in, size_t n, const uint32_t* perm
 // Grid structures (cd_options.grid_table): kOpen = the paper's open-addressing map with per-cell
 // lists, kChained = chained spatial hash, kCsr = open-addressing map of per-cell counts plus a
 // counting sort of the entries by cell (sort + segment: each cell's objects contiguous).
-enum GridKind : int { kOpen = 0, kChained = 1, kCsr = 2, kChainedBall = 3, kChainedLean = 4 };
+enum GridKind : int { kOpen = 0, kChained = 1, kCsr = 2, kChainedBall = 3, kChainedLean = 4, kChainedBallLean = 5 };
 // kChainedBall: the chained grid compiled for ball-mode scans only (the grid variant's hot
 // instance: the half-shell branch's code had cost its ball-mode scan 3 % -- 59.7 vs 61.6 us per
 // 1M-object step -- through register allocation)
 // kChainedLean: the half-shell chained scan without the shard band, slot map and raw counts
 // (test_pair<true>), chosen when none of them is active
-__host__ __device__ constexpr bool is_chained(int k) { return k == kChained || k == kChainedBall || k == kChainedLean; }
+__host__ __device__ constexpr bool is_chained(int k) { return k >= kChained && k != kCsr; }
 
 // CSR grid insert: claim the cell's slot (128-bit CAS from a stale slot to {key, tag | 1}) or
 // count the object into it (64-bit atomicAdd on the head word; count in the low 32 bits).
@@ -596,7 +596,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
     if (!cell_of(g, p, c, fr)) return;
     // own bucket: successors only, every pair once (by the later-inserted object)
     walk<kLean>(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
-    if (kLean || (!kBallOnly && g.halfshell)) {   // (the lean instance runs half-shell scans only)
+    if ((kLean && !kBallOnly) || (!kBallOnly && g.halfshell)) {   // (the lean half-shell instance runs half-shell scans only)
         // L < 2 g_c: the 13 half-shell neighbour cells (each unordered pair of cells of a 3x3x3
         // block once, as in do_scan), only the probed cell's entries (tag).  The 27 cells of a
         // 3x3x3 block differ pairwise in (c mod 4) on some axis, so with superblock buckets they
@@ -903,7 +903,7 @@ __global__ void __launch_bounds__(256, kGrid == kChained || kGrid == kChainedLea
         }
         if (r < a.O.n) {
             if (is_chained(kGrid))
-                do_scan_chained<kGrid == kChainedBall, kGrid == kChainedLean>(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
+                do_scan_chained<kGrid == kChainedBall || kGrid == kChainedBallLean, kGrid == kChainedLean || kGrid == kChainedBallLean>(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
                                 a.qcap, a.ctrl);
             else if (kGrid == kCsr)
                 do_scan_csr(a.g, a.scan_tab, a.scan_start, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r,
@@ -952,7 +952,7 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
         return launch_ex(k_step<kOpen, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
     }
     if (a.chained)
-        return launch_ex(!a.g.halfshell ? k_step<kChainedBall, 0>
+        return launch_ex(!a.g.halfshell ? (lean ? k_step<kChainedBallLean, 0> : k_step<kChainedBall, 0>)
                          : lean      ? k_step<kChainedLean, 0>
                                      : k_step<kChained, 0>,
                          dim3((unsigned)blocks),
