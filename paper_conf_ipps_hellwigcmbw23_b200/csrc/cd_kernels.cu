@@ -400,9 +400,10 @@ extern __shared__ Cand s_cand[];
 __shared__ unsigned s_nw[8];
 __shared__ unsigned s_rw[8];   // per warp: pairs examined (emit_raw_counts)
 
-// kLean: no radial shard band, no slot -> id map, no raw counts (the hybrid's default call; a
-// separate instance so these features cost it no registers)
-template <bool kLean = false>
+// kLean: no radial shard band, no slot -> id map, no raw counts (the default calls; separate
+// instances so these features cost them no registers); kLean == 2 also without candidate staging
+// (sparse ball-mode grids)
+template <int kLean = 0>
 __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_t j, const double p[3],
                                           const Entry& ej, uint32_t step, Cand* __restrict__ q,
                                           size_t qcap, Ctrl* ctrl)
@@ -423,7 +424,7 @@ __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_
         cd.i = a < b ? a : b;
         cd.j = a < b ? b : a;
         cd.step = step;
-        if (g.stage) {
+        if (kLean != 2 && g.stage) {
             const unsigned w = threadIdx.x >> 5;
             const unsigned k = atomicAdd(&s_nw[w], 1u);
             if (k < kSWarp) {
@@ -435,7 +436,7 @@ __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_
     }
 }
 
-template <bool kLean = false>
+template <int kLean = 0>
 __device__ __forceinline__ void walk(const GridGeom& g, const Entry* __restrict__ E, uint32_t j,
                                      uint32_t r, const double p[3], bool only_greater, uint32_t step,
                                      Cand* __restrict__ q, size_t qcap, Ctrl* ctrl)
@@ -557,7 +558,7 @@ __device__ __forceinline__ uint32_t head_index(uint32_t h, uint32_t epoch)
 // ball mode: bucket of the probed cell (tag ctag), which lies in the positive half-space of the
 // scanning object's cell -- only the probed cell's own entries count (a colliding neighbour
 // cell's entries are found by their own probe, so each pair is reported exactly once)
-template <bool kLean = false>
+template <int kLean = 0>
 __device__ __forceinline__ void walk_bucket_tag(const GridGeom& g, const Entry* __restrict__ E,
                                                 uint32_t h, uint32_t epoch, uint32_t ctag, uint32_t r,
                                                 const double p[3], uint32_t step,
@@ -582,6 +583,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
                                                 int s, int64_t r, uint32_t epoch, Cand* __restrict__ q,
                                                 size_t qcap, Ctrl* ctrl)
 {
+    constexpr int kTP = kLean ? (kBallOnly ? 2 : 1) : 0;   // test_pair flavour
     const uint32_t* heads = tab.bits + (size_t)s * tab.bwords;
     const uint32_t hmask = tab.bmask;
     const Entry* E = ents + (size_t)s * n;
@@ -595,7 +597,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
     double fr[3];
     if (!cell_of(g, p, c, fr)) return;
     // own bucket: successors only, every pair once (by the later-inserted object)
-    walk<kLean>(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
+    walk<kTP>(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
     if ((kLean && !kBallOnly) || (!kBallOnly && g.halfshell)) {   // (the lean half-shell instance runs half-shell scans only)
         // L < 2 g_c: the 13 half-shell neighbour cells (each unordered pair of cells of a 3x3x3
         // block once, as in do_scan), only the probed cell's entries (tag).  The 27 cells of a
@@ -617,7 +619,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
             const int o = __ffs(hit) - 1;
             hit &= hit - 1;
             const int cx = c[0] + kHalfShell[o][0], cy = c[1] + kHalfShell[o][1], cz = c[2] + kHalfShell[o][2];
-            walk_bucket_tag<kLean>(g, E, __ldg(heads + chain_bucket(cx, cy, cz, hmask)), epoch, cell_tag(cx, cy, cz),
+            walk_bucket_tag<kTP>(g, E, __ldg(heads + chain_bucket(cx, cy, cz, hmask)), epoch, cell_tag(cx, cy, cz),
                             (uint32_t)r, p, step, q, qcap, ctrl);
         }
         return;
@@ -644,7 +646,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
 #pragma unroll
     for (int b = 1; b < 8; ++b)
         if (hd[b])
-            walk_bucket_tag<kLean>(g, E, hd[b], epoch,
+            walk_bucket_tag<kTP>(g, E, hd[b], epoch,
                             cell_tag(c[0] + ((b & 1) ? d0 : 0), c[1] + ((b & 2) ? d1 : 0),
                                      c[2] + ((b & 4) ? d2 : 0)),
                             (uint32_t)r, p, step, q, qcap, ctrl);
@@ -892,9 +894,10 @@ __global__ void __launch_bounds__(256, kGrid == kChained || kGrid == kChainedLea
         if (a.scan_B == 0) return;
         const int s = (int)(b3 / nbC);
         const int64_t r = (int64_t)(b3 % nbC) * 256 + threadIdx.x;
-        const bool stage = a.g.stage != 0;   // uniform over the launch
+        const bool stage = kGrid != kChainedBallLean && a.g.stage != 0;   // uniform over the launch
+        const bool raw = kGrid != kChainedBallLean && kGrid != kChainedLean && a.g.raw;
         const unsigned lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-        if (stage || a.g.raw) {
+        if (stage || raw) {
             if (lane == 0) {
                 s_nw[wid] = 0;
                 s_rw[wid] = 0;
@@ -912,7 +915,7 @@ __global__ void __launch_bounds__(256, kGrid == kChained || kGrid == kChainedLea
                 do_scan(a.g, a.scan_tab, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r, a.scan_tag, a.q,
                         a.qcap, a.ctrl);
         }
-        if (a.g.raw) {
+        if (raw) {
             __syncwarp();
             if (lane == 0 && s_rw[wid]) atomicAdd(&a.ctrl->n_raw, (unsigned long long)s_rw[wid]);
         }
@@ -952,7 +955,7 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
         return launch_ex(k_step<kOpen, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
     }
     if (a.chained)
-        return launch_ex(!a.g.halfshell ? (lean ? k_step<kChainedBallLean, 0> : k_step<kChainedBall, 0>)
+        return launch_ex(!a.g.halfshell ? (lean && !a.g.stage ? k_step<kChainedBallLean, 0> : k_step<kChainedBall, 0>)
                          : lean      ? k_step<kChainedLean, 0>
                                      : k_step<kChained, 0>,
                          dim3((unsigned)blocks),
