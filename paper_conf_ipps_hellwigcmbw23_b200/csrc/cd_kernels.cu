@@ -268,12 +268,14 @@ cudaError_t launch_conj_to_global(const Conj* in, size_t n, const uint32_t* perm
 // Grid structures (cd_options.grid_table): kOpen = the paper's open-addressing map with per-cell
 // lists, kChained = chained spatial hash, kCsr = open-addressing map of per-cell counts plus a
 // counting sort of the entries by cell (sort + segment: each cell's objects contiguous).
-enum GridKind : int { kOpen = 0, kChained = 1, kCsr = 2, kChainedBall = 3, kChainedLean = 4, kChainedBallLean = 5 };
+enum GridKind : int { kOpen = 0, kChained = 1, kCsr = 2, kChainedBall = 3, kChainedLean = 4, kChainedBallLean = 5,
+                      kChainedBallLeanSig = 6 };
 // kChainedBall: the chained grid compiled for ball-mode scans only (the grid variant's hot
 // instance: the half-shell branch's code had cost its ball-mode scan 3 % -- 59.7 vs 61.6 us per
 // 1M-object step -- through register allocation)
-// kChainedLean: the half-shell chained scan without the shard band, slot map and raw counts
-// (test_pair<true>), chosen when none of them is active
+// kChainedLean / kChainedBallLean / kChainedBallLeanSig: the chained scans without the shard band
+// and raw counts (ball mode also without candidate staging; see test_pair's flavours), chosen
+// when none of those is active; kChainedLean without the spatial order's slot map
 __host__ __device__ constexpr bool is_chained(int k) { return k >= kChained && k != kCsr; }
 
 // CSR grid insert: claim the cell's slot (128-bit CAS from a stale slot to {key, tag | 1}) or
@@ -400,31 +402,34 @@ extern __shared__ Cand s_cand[];
 __shared__ unsigned s_nw[8];
 __shared__ unsigned s_rw[8];   // per warp: pairs examined (emit_raw_counts)
 
-// kLean: no radial shard band, no slot -> id map, no raw counts (the default calls; separate
-// instances so these features cost them no registers); kLean == 2 also without candidate staging
-// (sparse ball-mode grids)
+// test_pair flavours (bit flags; separate instances so the unused features cost no registers):
+// kTpLean = no radial shard band and no raw counts, kTpNoStage = no candidate staging (sparse
+// ball-mode grids), kTpSig = the slot -> id map of the spatial order (lean instances only; the
+// full one reads it at run time)
+constexpr int kTpLean = 1, kTpNoStage = 2, kTpSig = 4;
 template <int kLean = 0>
 __device__ __forceinline__ void test_pair(const GridGeom& g, uint32_t r, uint32_t j, const double p[3],
                                           const Entry& ej, uint32_t step, Cand* __restrict__ q,
                                           size_t qcap, Ctrl* ctrl)
 {
-    if (!kLean && g.raw) atomicAdd(&s_rw[threadIdx.x >> 5], 1u);
+    if (!(kLean & kTpLean) && g.raw) atomicAdd(&s_rw[threadIdx.x >> 5], 1u);
     const double dx = p[0] - ej.x, dy = p[1] - ej.y, dz = p[2] - ej.z;
     if (fma(dx, dx, fma(dy, dy, dz * dz)) < g.gc2) {
         // radial shard: the pair belongs to the shard holding the smaller radius (identical
         // positions on every shard, so exactly one shard keeps it)
-        if (!kLean) {
+        if (!(kLean & kTpLean)) {
             const double ra = fma(p[0], p[0], fma(p[1], p[1], p[2] * p[2]));
             const double rb = fma(ej.x, ej.x, fma(ej.y, ej.y, ej.z * ej.z));
             const double rm = fmin(ra, rb);
             if (!(rm >= g.band_lo2 && rm < g.band_hi2)) return;
         }
-        const uint32_t a = !kLean && g.sig ? g.sig[r] : r, b = !kLean && g.sig ? g.sig[j] : j;   // slots -> internal ids
+        constexpr bool kSigRt = !(kLean & kTpLean) || (kLean & kTpSig);   // slots -> internal ids
+        const uint32_t a = kSigRt && g.sig ? g.sig[r] : r, b = kSigRt && g.sig ? g.sig[j] : j;
         Cand cd;
         cd.i = a < b ? a : b;
         cd.j = a < b ? b : a;
         cd.step = step;
-        if (kLean != 2 && g.stage) {
+        if (!(kLean & kTpNoStage) && g.stage) {
             const unsigned w = threadIdx.x >> 5;
             const unsigned k = atomicAdd(&s_nw[w], 1u);
             if (k < kSWarp) {
@@ -577,13 +582,12 @@ __device__ __forceinline__ void walk_bucket_tag(const GridGeom& g, const Entry* 
     }
 }
 
-template <bool kBallOnly, bool kLean = false>
+template <bool kBallOnly, int kTP = 0>
 __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab& tab,
                                                 const Entry* __restrict__ ents, int64_t n, int64_t k0,
                                                 int s, int64_t r, uint32_t epoch, Cand* __restrict__ q,
                                                 size_t qcap, Ctrl* ctrl)
 {
-    constexpr int kTP = kLean ? (kBallOnly ? 2 : 1) : 0;   // test_pair flavour
     const uint32_t* heads = tab.bits + (size_t)s * tab.bwords;
     const uint32_t hmask = tab.bmask;
     const Entry* E = ents + (size_t)s * n;
@@ -598,7 +602,7 @@ __device__ __forceinline__ void do_scan_chained(const GridGeom& g, const GridTab
     if (!cell_of(g, p, c, fr)) return;
     // own bucket: successors only, every pair once (by the later-inserted object)
     walk<kTP>(g, E, me.next, (uint32_t)r, p, false, step, q, qcap, ctrl);
-    if ((kLean && !kBallOnly) || (!kBallOnly && g.halfshell)) {   // (the lean half-shell instance runs half-shell scans only)
+    if (((kTP & kTpLean) && !kBallOnly) || (!kBallOnly && g.halfshell)) {   // (the lean half-shell instance runs half-shell scans only)
         // L < 2 g_c: the 13 half-shell neighbour cells (each unordered pair of cells of a 3x3x3
         // block once, as in do_scan), only the probed cell's entries (tag).  The 27 cells of a
         // 3x3x3 block differ pairwise in (c mod 4) on some axis, so with superblock buckets they
@@ -894,8 +898,11 @@ __global__ void __launch_bounds__(256, kGrid == kChained || kGrid == kChainedLea
         if (a.scan_B == 0) return;
         const int s = (int)(b3 / nbC);
         const int64_t r = (int64_t)(b3 % nbC) * 256 + threadIdx.x;
-        const bool stage = kGrid != kChainedBallLean && a.g.stage != 0;   // uniform over the launch
-        const bool raw = kGrid != kChainedBallLean && kGrid != kChainedLean && a.g.raw;
+        constexpr int kTP = kGrid == kChainedLean ? kTpLean
+                            : kGrid == kChainedBallLean ? kTpLean | kTpNoStage
+                            : kGrid == kChainedBallLeanSig ? kTpLean | kTpNoStage | kTpSig : 0;
+        const bool stage = !(kTP & kTpNoStage) && a.g.stage != 0;   // uniform over the launch
+        const bool raw = !(kTP & kTpLean) && a.g.raw;
         const unsigned lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
         if (stage || raw) {
             if (lane == 0) {
@@ -906,7 +913,7 @@ __global__ void __launch_bounds__(256, kGrid == kChained || kGrid == kChainedLea
         }
         if (r < a.O.n) {
             if (is_chained(kGrid))
-                do_scan_chained<kGrid == kChainedBall || kGrid == kChainedBallLean, kGrid == kChainedLean || kGrid == kChainedBallLean>(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
+                do_scan_chained<kGrid == kChainedBall || kGrid == kChainedBallLean || kGrid == kChainedBallLeanSig, kTP>(a.g, a.scan_tab, a.scan_ents, a.O.n, a.scan_k0, s, r, a.scan_tag, a.q,
                                 a.qcap, a.ctrl);
             else if (kGrid == kCsr)
                 do_scan_csr(a.g, a.scan_tab, a.scan_start, a.scan_ents, a.O.n, a.mask, a.scan_k0, s, r,
@@ -945,7 +952,7 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
     if (blocks == 0) return cudaSuccess;
     lc.bump();
     const size_t smem = a.g.stage ? sizeof(Cand) * kSCand : 0;   // candidate staging buffer
-    const bool lean = !a.g.raw && !a.g.sig && a.g.band_lo2 == 0.0 && isinf(a.g.band_hi2);
+    const bool lean = !a.g.raw && a.g.band_lo2 == 0.0 && isinf(a.g.band_hi2);   // (no shard band, no raw counts)
     if (a.O.j2) {   // J2 secular propagator: the rotation is compiled into its own instances
         if (a.chained)
             return launch_ex(a.g.halfshell ? k_step<kChained, 1> : k_step<kChainedBall, 1>, dim3((unsigned)blocks),
@@ -955,8 +962,9 @@ cudaError_t launch_step(StepArgs a, const L2Win* win, cudaStream_t st, LaunchCou
         return launch_ex(k_step<kOpen, 1>, dim3((unsigned)blocks), dim3(256), smem, st, win, false, a);
     }
     if (a.chained)
-        return launch_ex(!a.g.halfshell ? (lean && !a.g.stage ? k_step<kChainedBallLean, 0> : k_step<kChainedBall, 0>)
-                         : lean      ? k_step<kChainedLean, 0>
+        return launch_ex(!a.g.halfshell ? (lean && !a.g.stage ? (a.g.sig ? k_step<kChainedBallLeanSig, 0> : k_step<kChainedBallLean, 0>)
+                                                               : k_step<kChainedBall, 0>)
+                         : lean && !a.g.sig ? k_step<kChainedLean, 0>
                                      : k_step<kChained, 0>,
                          dim3((unsigned)blocks),
                          dim3(256), smem, st, win, a.pdl != 0, a);
