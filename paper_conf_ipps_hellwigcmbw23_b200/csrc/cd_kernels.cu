@@ -857,7 +857,13 @@ template <int kGrid, int kJ2>
 #ifndef CD_HALF_MINB
 #define CD_HALF_MINB 8   // kChained: the half-shell (and J2 runtime) instance
 #endif
+// the lean ball instance (the 1M grid's) at 7 blocks per SM: 56.2 -> 53.3 us per step (8: 53.4);
+// the lean instance with the slot map (8M, spatial order) stays at 6 (7: 766 vs 738 us)
+#ifndef CD_BALL_LEAN_MINB
+#define CD_BALL_LEAN_MINB 7
+#endif
 __global__ void __launch_bounds__(256, kGrid == kChained || kGrid == kChainedLean ? CD_HALF_MINB
+                                       : kGrid == kChainedBallLean ? CD_BALL_LEAN_MINB
                                        : is_chained(kGrid) ? CD_STEP_MINB
                                        : kGrid == kCsr     ? CD_CSR_MINB
                                                            : CD_OPEN_MINB) k_step(StepArgs a)
