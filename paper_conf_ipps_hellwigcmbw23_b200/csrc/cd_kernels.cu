@@ -853,15 +853,15 @@ __device__ __forceinline__ void do_scan_csr(const GridGeom& g, const GridTab& ta
 #ifndef CD_CSR_MINB
 #define CD_CSR_MINB 6
 #endif
-template <int kGrid, int kJ2>
 #ifndef CD_HALF_MINB
-#define CD_HALF_MINB 8   // kChained: the half-shell (and J2 runtime) instance
+#define CD_HALF_MINB 8   // kChained / kChainedLean: the half-shell (and J2 runtime) instances
 #endif
 // the lean ball instance (the 1M grid's) at 7 blocks per SM: 56.2 -> 53.3 us per step (8: 53.4);
 // the lean instance with the slot map (8M, spatial order) stays at 6 (7: 766 vs 738 us)
 #ifndef CD_BALL_LEAN_MINB
 #define CD_BALL_LEAN_MINB 7
 #endif
+template <int kGrid, int kJ2>
 __global__ void __launch_bounds__(256, kGrid == kChained || kGrid == kChainedLean ? CD_HALF_MINB
                                        : kGrid == kChainedBallLean ? CD_BALL_LEAN_MINB
                                        : is_chained(kGrid) ? CD_STEP_MINB
